@@ -1,0 +1,374 @@
+#!/usr/bin/env python
+"""Benchmark: BC traversal rate (GTEPS = m x sources / s) on N B200s.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c4] [--impl ours|reference]
+
+One STEP = one complete betweenness-centrality computation of the workload's
+source set (all of SURVEY §8(a): Alg. 5 sampling phase, decision, forward +
+backward traversal of every source, BC accumulation, halving) plus, for N > 1,
+the single NCCL all-reduce of the per-GPU BC vectors.  The default
+workload is configs[3] of BASELINE.json -- Graph500 Kronecker scale 18, edge
+factor 16, 16,384 sources -- the configuration the metric is quoted on at
+1/2/4/8 GPUs.  Scaling is weak: every rank processes 16,384 sources of its own
+(--scaling strong splits one 16,384-source set instead).
+
+Timing: inputs resident in HBM; L2 flushed (256 MiB write)
+before every timed step; CUDA events on the launching stream; barrier +
+synchronize on both sides; max over ranks.  `e2e` repeats the measurement
+through the host-buffer C-ABI call bc_compute (host sources in, host BC out).
+`roofline` uses the algorithmic byte model of SURVEY §8(d) with the per-source
+counts returned by the kernel, against MEASURED_PEAKS.json's HBM bandwidth.
+`cpu_baseline` (and --impl reference) time the CPU oracle on this host.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "BC traversal GTEPS (m×sources/s) at 1/2/4/8 B200; % of HBM roofline"
+UNIT = "GTEPS"
+
+
+def log(*a):
+    print("[bench]", *a, file=sys.stderr, flush=True)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+# ---------------------------------------------------------------- workload
+
+
+def make_workload(cfg_key: str, world: int, rank: int, scaling: str):
+    from paper_conf_sc_mclaughlinb14_b200 import graphgen as gg
+    from paper_conf_sc_mclaughlinb14_b200.distributed import shard_sources
+    cfg = gg.CONFIGS[cfg_key]
+    g = cfg.graph()
+    if cfg.k is None:                     # exact BC: all vertices
+        total = np.arange(g.n, dtype=np.int32)
+        local = shard_sources(total, rank, world, seed=cfg.seed)
+        per_rank = None
+    elif scaling == "weak":
+        per_rank = cfg.k
+        total = gg.sample_sources(g, min(cfg.k * world, int((g.degrees() > 0).sum())), cfg.seed + 7)
+        local = shard_sources(total, rank, world, seed=cfg.seed)
+    else:
+        total = cfg.sources(g)
+        local = shard_sources(total, rank, world, seed=cfg.seed)
+        per_rank = None
+    return cfg, g, total, local
+
+
+# ---------------------------------------------------------------- clocks
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons (NVML) while the timed region runs."""
+
+    def __init__(self, dev_index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+        except Exception as e:  # pragma: no cover - no NVML
+            log("NVML unavailable:", e)
+            self.nv = None
+
+    def _run(self):
+        nv = self.nv
+        names = {
+            "hw_slowdown": getattr(nv, "nvmlClocksEventReasonHwSlowdown", 0x8),
+            "hw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
+            "sw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
+            "sw_power_cap": getattr(nv, "nvmlClocksEventReasonSwPowerCap", 0x4),
+            "hw_power_brake_slowdown": getattr(nv, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
+        }
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for k, bit in names.items():
+                    if r & bit:
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            self._stop.wait(0.05)
+
+    def __enter__(self):
+        if self.nv:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.nv:
+            self.t.join()
+
+    def summary(self):
+        return {"sm_mhz": statistics.median(self.samples) if self.samples else None,
+                "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+# ---------------------------------------------------------------- CPU oracle
+
+
+def time_oracle(g, sources, budget_s: float, nthreads: int):
+    """Time the oracle on a bounded prefix of `sources` sized to ~budget_s."""
+    import oracle
+    oracle.build()
+    probe = sources[: max(4, min(32, sources.size))]
+    t0 = time.perf_counter()
+    oracle.bc(g, probe, nthreads=nthreads)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    k = int(min(sources.size, max(probe.size, probe.size * budget_s / dt)))
+    k = max(nthreads, (k // nthreads) * nthreads) if k >= nthreads else k
+    sample = sources[:k]
+    t0 = time.perf_counter()
+    oracle.bc(g, sample, nthreads=nthreads)
+    dt = time.perf_counter() - t0
+    return g.m * k / dt / 1e9, k, dt
+
+
+# ---------------------------------------------------------------- arms
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, on this host's cores."""
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    cfg, g, total, _ = make_workload(args.config, world, 0, args.scaling)
+    cores = len(os.sched_getaffinity(0))
+    per_step = max(5.0, 150.0 / max(1, args.steps + args.warmup))
+    import oracle
+    oracle.build()
+    # calibrate the per-step sample to ~per_step seconds on all cores
+    _, k, _ = time_oracle(g, total, min(per_step, 5.0), cores)
+    k = int(min(total.size, max(cores, k * per_step / min(per_step, 5.0))))
+    sample = total[:k]
+    for _ in range(args.warmup):
+        oracle.bc(g, sample[: max(1, k // 8)], nthreads=cores)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.bc(g, sample, nthreads=cores)
+        times.append(time.perf_counter() - t0)
+    T = sum(times)
+    value = g.m * k * args.steps / T / 1e9
+    desc = f"first {k} of the workload's {total.size} sources per step, {cores} threads"
+    out = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * T / args.steps,
+        "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic", "config": workload_config(cfg, g, total, world, args),
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": desc},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def workload_config(cfg, g, total, world, args):
+    return {"workload": f"{cfg.key}: {cfg.description}", "graph": g.name, "n": g.n, "m": g.m,
+            "sources_total": int(total.size), "sources_per_gpu": int(math.ceil(total.size / world)),
+            "strategy": args.strategy, "parallelism": f"sources split over {world} GPU(s)",
+            "l2": "flushed before every timed step (256 MiB write)", "seed": cfg.seed}
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_mclaughlinb14_b200 as bcm
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        log(f"WORLD_SIZE={world} but --gpus {args.gpus}; using WORLD_SIZE")
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    t0 = time.time()
+    cfg, g, total, local = make_workload(args.config, world, rank, args.scaling)
+    log(f"rank {rank}: graph {g.name} n={g.n} m={g.m} local sources {local.size} "
+        f"(gen {time.time() - t0:.1f}s)")
+    bg = bcm.BCGraph.from_graph(g, device=local_rank, strategy=args.strategy)
+    stream = torch.cuda.Stream(dev)
+    d_src = torch.from_numpy(local).to(dev)
+    out = torch.zeros(g.n, dtype=torch.float64, device=dev)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def step():
+        with torch.cuda.stream(stream):
+            bg.compute_device(d_src, out, stream=stream)
+            if world > 1:
+                dist.all_reduce(out)
+
+    def barrier():
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier(device_ids=[local_rank])
+
+    for _ in range(args.warmup):
+        step()
+    barrier()
+
+    hbm, hbm_src = peaks()
+    step_ms, kern_ms, bytes_alg, launches, bc_launches = [], [], [], 0, 0
+    st = None
+    with ClockSampler(local_rank) as clk:
+        for _ in range(args.steps):
+            flush.fill_(1)                           # evict L2 between timed steps
+            barrier()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            step()
+            e1.record(stream)
+            barrier()
+            step_ms.append(e0.elapsed_time(e1))
+            st = bg.stats()                          # outside the events
+            kern_ms.append(st["kernel_ms"])
+            launches += st["kernel_launches"]
+            bc_launches += st["bc_kernel_launches"]
+            # B(s) = 20 n + 16 A_R + 24 D + 64 n_R per source
+            bytes_alg.append(20.0 * g.n * st["sources"] + 16.0 * st["arcs_reached"]
+                             + 24.0 * st["dag_arcs"] + 64.0 * st["n_reached"])
+    T_local = sum(step_ms) / 1e3
+    T = torch.tensor([T_local], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(T, op=dist.ReduceOp.MAX)
+    T = float(T.item())
+    value = g.m * total.size * args.steps / T / 1e9
+
+    # -------- e2e: host-buffer C-ABI call (sources H2D and BC D2H inside the region)
+    host_src = torch.from_numpy(local).pin_memory()
+    host_bc = torch.empty(g.n, dtype=torch.float64).pin_memory()
+    e2e_ms = []
+    for it in range(args.warmup + args.steps):
+        flush.fill_(1)
+        barrier()
+        t0 = time.perf_counter()
+        bcm.bc_compute(bg.handle, host_src.numpy(), host_bc.numpy())
+        if world > 1:
+            dv = host_bc.to(dev, non_blocking=True)
+            dist.all_reduce(dv)
+            host_bc.copy_(dv)
+            torch.cuda.synchronize(dev)
+        t1 = time.perf_counter()
+        if it >= args.warmup:
+            e2e_ms.append((t1 - t0) * 1e3)
+    Te = torch.tensor([sum(e2e_ms) / 1e3], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(Te, op=dist.ReduceOp.MAX)
+    e2e_value = g.m * total.size * args.steps / float(Te.item()) / 1e9
+    h2d = 4 * local.size + (8 * g.n if world > 1 else 0)
+    d2h = 8 * g.n * (2 if world > 1 else 1)
+
+    # -------- roofline of the dominant kernel (bc_kernel): algorithmic bytes / its event time
+    kms = sum(kern_ms) / max(1, len(kern_ms))
+    balg = sum(bytes_alg) / max(1, len(bytes_alg))
+    achieved = balg / (kms / 1e3) / 1e9 if kms > 0 else 0.0
+    traffic = load_traffic(args.config, balg, st)
+    roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+            "frac": achieved / hbm, "traffic": traffic, "peak_source": hbm_src,
+            "kernel": "bc_kernel (sampling + main launches per step)",
+            "kernel_ms_per_step": kms, "kernel_share_of_step": kms / (sum(step_ms) / len(step_ms)),
+            "alg_bytes_per_step": balg,
+            "alg_bytes_per_teps_edge": balg / (g.m * st["sources"]) if st and st["sources"] else None,
+            "model": "SURVEY 8(d): B(s) = 20n + 16 A_R + 24 D + 64 n_R per source"}
+
+    result = None
+    if rank == 0:
+        cores = len(os.sched_getaffinity(0))
+        cpu = None
+        if not args.no_cpu_baseline and world == 1:
+            v, k, dt = time_oracle(g, local, args.cpu_budget, cores)
+            cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+                   "sample": f"first {k} of the {local.size} workload sources ({dt:.1f}s on {cores} threads)"}
+        result = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * T / args.steps, "higher_is_better": True,
+            "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": workload_config(cfg, g, total, world, args),
+            "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+                    "d2h_bytes_per_step": int(d2h)},
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "clocks": clk.summary(),
+            "gpu_launches": int(launches),
+            "stats": {k2: st[k2] for k2 in ("sources", "levels", "we_levels", "ep_levels",
+                                            "sampling_ep", "sampling_median", "inflight",
+                                            "sigma_inexact", "arcs_scanned", "n_reached",
+                                            "arcs_reached", "dag_arcs")},
+            "paper_context": "398.63 MTEPS on 1x GTX Titan (Table III, smallworld); 24.13 GTEPS on "
+                             "192x Tesla M2090 (Table IV, kron_g500-logn20)",
+        }
+        print(json.dumps(result), flush=True)
+    bg.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def load_traffic(cfg_key, balg, st):
+    """DRAM bytes per launch-step from the committed ncu capture, scaled by the
+    algorithmic bytes (profiles/traffic.json: dram bytes per algorithmic byte)."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        d = json.load(open(p)).get(cfg_key)
+        return None if d is None else d["dram_bytes_per_alg_byte"] * balg
+    except Exception:
+        return None
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c4")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--strategy", default="sampling", choices=["we", "ep", "hybrid", "sampling"])
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        log("warmup < 3 is not allowed by the timing rules; using 3")
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

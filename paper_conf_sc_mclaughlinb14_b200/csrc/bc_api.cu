@@ -1,0 +1,549 @@
+// bc_api.cu -- host side of libbc.so: the C ABI declared in include/bc.h.
+//
+// Graph ingest, workspace sizing, the launch sequence of one
+// bc_compute (sampling phase -> decision -> main phase -> halving, Alg. 5
+// P:283-301), stats and errors.  All arithmetic of the method runs in the
+// kernels of bc_kernels.cuh; this file only validates, copies and launches.
+#include "bc.h"
+#include "bc_kernels.cuh"
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+using namespace bcdev;
+
+namespace {
+
+thread_local char g_err[512] = "";
+
+int fail(int code, const char *fmt, ...) {
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(g_err, sizeof(g_err), fmt, ap);
+    va_end(ap);
+    return code;
+}
+
+#define CK(call)                                                                         \
+    do {                                                                                 \
+        cudaError_t e_ = (call);                                                         \
+        if (e_ != cudaSuccess)                                                           \
+            return fail(e_ == cudaErrorMemoryAllocation ? BC_ENOMEM : BC_ECUDA,          \
+                        "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, \
+                        __LINE__);                                                       \
+    } while (0)
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        cudaGetDevice(&prev);
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur;
+        if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+}  // namespace
+
+struct bc_graph {
+    int device = 0;
+    int n = 0;
+    int nnz = 0;
+    int directed = 0;
+    int num_sms = 0;
+    int occ_slots = 0;  // occupancy-limited CTA count
+    // graph
+    int *ro = nullptr, *col = nullptr, *src = nullptr;
+    int *iro = nullptr, *icol = nullptr, *isrc = nullptr;
+    // workspace
+    int slots = 0;
+    int *d = nullptr;
+    double *sigma = nullptr, *omega = nullptr;
+    int *S = nullptr, *ends = nullptr;
+    unsigned char *modes = nullptr;
+    size_t stride_n = 0, stride_e = 0;
+    // per-call buffers
+    int *src_buf = nullptr;
+    long long src_cap = 0;
+    double *bc_buf = nullptr;
+    unsigned long long *counters = nullptr;  // [0] sampling phase, [1] main phase
+    int *keys = nullptr;
+    int *flag = nullptr;                     // Alg. 5 decision (persists for single-source)
+    DevStats *stats = nullptr;
+    cudaStream_t stream = nullptr;           // own stream for the host-buffer API
+    cudaEvent_t done = nullptr;              // end of the last enqueued call
+    bc_options opt{};
+    int sampling_ran = 0;
+    int last_inflight = 0;
+    int launches = 0;        // kernels launched by the last compute call
+    int bc_launches = 0;     // ... of which bc_kernel
+    cudaEvent_t tev[4] = {nullptr, nullptr, nullptr, nullptr};  // around the bc_kernel launches
+    int tev_used[2] = {0, 0};
+};
+
+extern "C" void bc_default_options(bc_options *o) {
+    if (!o) return;
+    o->strategy = BC_STRATEGY_SAMPLING;
+    o->alpha = 768;
+    o->beta = 512;
+    o->gamma = 4.0;
+    o->n_samps = 512;
+    o->ep_min_frontier = 512;
+    o->inflight = 0;
+    o->backward_we = 0;
+}
+
+extern "C" const char *bc_last_error(void) { return g_err; }
+
+static void free_workspace(bc_graph *g) {
+    cudaFree(g->d);
+    cudaFree(g->sigma);
+    cudaFree(g->omega);
+    cudaFree(g->S);
+    cudaFree(g->ends);
+    cudaFree(g->modes);
+    g->d = nullptr;
+    g->sigma = g->omega = nullptr;
+    g->S = g->ends = nullptr;
+    g->modes = nullptr;
+    g->slots = 0;
+}
+
+static size_t slot_bytes(const bc_graph *g) {
+    return g->stride_n * (sizeof(int) + 2 * sizeof(double) + sizeof(int)) +
+           g->stride_e * (sizeof(int) + 1);
+}
+
+static int alloc_workspace(bc_graph *g) {
+    free_workspace(g);
+    g->stride_n = (size_t)std::max(g->n, 1);
+    g->stride_n = (g->stride_n + 31) & ~(size_t)31;  // 128-byte aligned slots
+    g->stride_e = g->stride_n + 32;
+    int want = g->opt.inflight > 0 ? std::min(g->opt.inflight, g->occ_slots) : g->occ_slots;
+    size_t free_b = 0, total_b = 0;
+    CK(cudaMemGetInfo(&free_b, &total_b));
+    size_t per = slot_bytes(g);
+    size_t budget = (size_t)(0.6 * (double)free_b);
+    int cap = (int)std::max<size_t>(1, budget / std::max<size_t>(per, 1));
+    g->slots = std::max(1, std::min(want, cap));
+    size_t ns = (size_t)g->slots;
+    CK(cudaMalloc(&g->d, ns * g->stride_n * sizeof(int)));
+    CK(cudaMalloc(&g->sigma, ns * g->stride_n * sizeof(double)));
+    CK(cudaMalloc(&g->omega, ns * g->stride_n * sizeof(double)));
+    CK(cudaMalloc(&g->S, ns * g->stride_n * sizeof(int)));
+    CK(cudaMalloc(&g->ends, ns * g->stride_e * sizeof(int)));
+    CK(cudaMalloc(&g->modes, ns * g->stride_e));
+    CK(cudaMemset(g->d, 0x7F, ns * g->stride_n * sizeof(int)));  // INF = 0x7F7F7F7F
+    CK(cudaMemset(g->sigma, 0, ns * g->stride_n * sizeof(double)));
+    CK(cudaMemset(g->omega, 0, ns * g->stride_n * sizeof(double)));
+    CK(cudaDeviceSynchronize());
+    return BC_OK;
+}
+
+extern "C" void bc_destroy(bc_graph *g) {
+    if (!g) return;
+    DeviceGuard dg(g->device);
+    if (g->done) cudaEventSynchronize(g->done);
+    free_workspace(g);
+    cudaFree(g->ro);
+    cudaFree(g->col);
+    cudaFree(g->src);
+    cudaFree(g->iro);
+    cudaFree(g->icol);
+    cudaFree(g->isrc);
+    cudaFree(g->src_buf);
+    cudaFree(g->bc_buf);
+    cudaFree(g->counters);
+    cudaFree(g->keys);
+    cudaFree(g->flag);
+    cudaFree(g->stats);
+    if (g->done) cudaEventDestroy(g->done);
+    for (auto &e : g->tev)
+        if (e) cudaEventDestroy(e);
+    if (g->stream) cudaStreamDestroy(g->stream);
+    delete g;
+}
+
+static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col) {
+    const int n = g->n;
+    const int nnz = g->nnz;
+    std::vector<int> ro32((size_t)n + 1);
+    for (int v = 0; v <= n; ++v) ro32[v] = (int)ro64[v];
+    CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&g->done, cudaEventDisableTiming));
+    for (auto &e : g->tev) CK(cudaEventCreate(&e));
+    CK(cudaMalloc(&g->ro, sizeof(int) * ((size_t)n + 1)));
+    CK(cudaMalloc(&g->col, sizeof(int) * (size_t)std::max(nnz, 1)));
+    CK(cudaMalloc(&g->src, sizeof(int) * (size_t)std::max(nnz, 1)));
+    CK(cudaMemcpy(g->ro, ro32.data(), sizeof(int) * ((size_t)n + 1), cudaMemcpyHostToDevice));
+    if (nnz) CK(cudaMemcpy(g->col, col, sizeof(int) * (size_t)nnz, cudaMemcpyHostToDevice));
+    if (nnz && n) {
+        build_src_kernel<<<std::min((nnz + 255) / 256, 148 * 16), 256>>>(g->ro, n, nnz, g->src);
+        CK(cudaGetLastError());
+    }
+    if (g->directed) {
+        // transpose on the host (counting sort keeps in-rows in ascending source order)
+        std::vector<int> iro((size_t)n + 1, 0), icol((size_t)std::max(nnz, 1)), fill((size_t)n);
+        for (int e = 0; e < nnz; ++e) iro[col[e] + 1]++;
+        for (int v = 0; v < n; ++v) iro[v + 1] += iro[v];
+        for (int v = 0; v < n; ++v) fill[v] = iro[v];
+        for (int u = 0; u < n; ++u)
+            for (int e = ro32[u]; e < ro32[u + 1]; ++e) icol[fill[col[e]]++] = u;
+        CK(cudaMalloc(&g->iro, sizeof(int) * ((size_t)n + 1)));
+        CK(cudaMalloc(&g->icol, sizeof(int) * (size_t)std::max(nnz, 1)));
+        CK(cudaMalloc(&g->isrc, sizeof(int) * (size_t)std::max(nnz, 1)));
+        CK(cudaMemcpy(g->iro, iro.data(), sizeof(int) * ((size_t)n + 1), cudaMemcpyHostToDevice));
+        if (nnz) {
+            CK(cudaMemcpy(g->icol, icol.data(), sizeof(int) * (size_t)nnz, cudaMemcpyHostToDevice));
+            build_src_kernel<<<std::min((nnz + 255) / 256, 148 * 16), 256>>>(g->iro, n, nnz, g->isrc);
+            CK(cudaGetLastError());
+        }
+    }
+    CK(cudaMalloc(&g->counters, 2 * sizeof(unsigned long long)));
+    CK(cudaMalloc(&g->keys, sizeof(int) * 8192));
+    CK(cudaMalloc(&g->flag, sizeof(int)));
+    CK(cudaMemset(g->flag, 0, sizeof(int)));
+    CK(cudaMalloc(&g->stats, sizeof(DevStats)));
+    CK(cudaMemset(g->stats, 0, sizeof(DevStats)));
+    CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
+    int per_sm = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+        &per_sm, g->directed ? (const void *)bc_kernel<true> : (const void *)bc_kernel<false>, NT, 0));
+    g->occ_slots = std::max(1, per_sm) * g->num_sms;
+    bc_default_options(&g->opt);
+    int rc = alloc_workspace(g);
+    if (rc) return rc;
+    CK(cudaDeviceSynchronize());
+    return BC_OK;
+}
+
+extern "C" int bc_graph_create(int32_t n, int64_t nnz, const int64_t *row_offsets,
+                               const int32_t *col_indices, int directed, int device,
+                               bc_graph **out) {
+    if (!out) return fail(BC_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (n < 0 || n > 0x7FFFFFFF - 64) return fail(BC_EINVAL, "n=%d out of range", n);
+    if (nnz < 0 || nnz > 0x7FFFFFFFLL - 1) return fail(BC_EINVAL, "nnz=%lld out of range (< 2^31)", (long long)nnz);
+    if (!row_offsets) return fail(BC_EINVAL, "row_offsets is NULL");
+    if (nnz > 0 && !col_indices) return fail(BC_EINVAL, "col_indices is NULL");
+    if (row_offsets[0] != 0) return fail(BC_EINVAL, "row_offsets[0] != 0");
+    if (row_offsets[n] != nnz) return fail(BC_EINVAL, "row_offsets[n]=%lld != nnz=%lld",
+                                           (long long)row_offsets[n], (long long)nnz);
+    for (int v = 0; v < n; ++v)
+        if (row_offsets[v + 1] < row_offsets[v])
+            return fail(BC_EINVAL, "row_offsets decreases at vertex %d", v);
+    for (int64_t e = 0; e < nnz; ++e)
+        if (col_indices[e] < 0 || col_indices[e] >= n)
+            return fail(BC_EINVAL, "col_indices[%lld]=%d out of range", (long long)e, col_indices[e]);
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+        return fail(BC_ECUDA, "no CUDA device available");
+    if (device < 0 || device >= ndev) return fail(BC_EINVAL, "device %d out of range", device);
+    bc_graph *g = new (std::nothrow) bc_graph();
+    if (!g) return fail(BC_ENOMEM, "host allocation failed");
+    g->device = device;
+    g->n = n;
+    g->nnz = (int)nnz;
+    g->directed = directed ? 1 : 0;
+    DeviceGuard dg(device);
+    int rc = create_impl(g, row_offsets, col_indices);
+    if (rc) {
+        bc_destroy(g);
+        return rc;
+    }
+    *out = g;
+    g_err[0] = 0;
+    return BC_OK;
+}
+
+extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
+    if (!g || !o) return fail(BC_EINVAL, "NULL argument");
+    if (o->strategy < 0 || o->strategy > 3) return fail(BC_EINVAL, "bad strategy %d", o->strategy);
+    if (o->n_samps < 1 || o->n_samps > 8192) return fail(BC_EINVAL, "n_samps must be in [1, 8192]");
+    if (o->alpha < 0 || o->beta < 0 || o->ep_min_frontier < 0 || o->inflight < 0 || !(o->gamma >= 0))
+        return fail(BC_EINVAL, "negative parameter");
+    DeviceGuard dg(g->device);
+    if (g->done) CK(cudaEventSynchronize(g->done));
+    const int realloc = o->inflight != g->opt.inflight;
+    g->opt = *o;
+    if (realloc) return alloc_workspace(g);
+    return BC_OK;
+}
+
+extern "C" int bc_get_options(const bc_graph *g, bc_options *o) {
+    if (!g || !o) return fail(BC_EINVAL, "NULL argument");
+    *o = g->opt;
+    return BC_OK;
+}
+
+static KParams base_params(bc_graph *g, double *d_bc) {
+    KParams p;
+    memset(&p, 0, sizeof(p));
+    p.n = g->n;
+    p.nnz = g->nnz;
+    p.ro = g->ro;
+    p.col = g->col;
+    p.src = g->src;
+    p.iro = g->directed ? g->iro : g->ro;
+    p.icol = g->directed ? g->icol : g->col;
+    p.isrc = g->directed ? g->isrc : g->src;
+    p.d = g->d;
+    p.sigma = g->sigma;
+    p.omega = g->omega;
+    p.S = g->S;
+    p.ends = g->ends;
+    p.modes = g->modes;
+    p.stride_n = g->stride_n;
+    p.stride_e = g->stride_e;
+    p.bc = d_bc;
+    p.alpha = g->opt.alpha;
+    p.beta = g->opt.beta;
+    p.ep_min_frontier = g->opt.ep_min_frontier;
+    p.backward_we = g->opt.backward_we;
+    p.stats = g->stats;
+    p.sampled_flag = g->flag;
+    return p;
+}
+
+static int launch(bc_graph *g, const KParams &p, cudaStream_t st) {
+    if (p.k <= 0) return BC_OK;
+    int grid = (int)std::min<long long>(g->slots, p.k);
+    if (g->directed) bc_kernel<true><<<grid, NT, 0, st>>>(p);
+    else bc_kernel<false><<<grid, NT, 0, st>>>(p);
+    g->last_inflight = std::max(g->last_inflight, grid);
+    g->launches++;
+    g->bc_launches++;
+    CK(cudaGetLastError());
+    return BC_OK;
+}
+
+// Enqueue one full BC computation on `st`.  d_sources may be NULL (all n).
+static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, double *d_bc,
+                           cudaStream_t st) {
+    CK(cudaStreamWaitEvent(st, g->done, 0));
+    g->sampling_ran = 0;
+    if (g->n == 0) {
+        CK(cudaMemsetAsync(g->stats, 0, sizeof(DevStats), st));
+        CK(cudaEventRecord(g->done, st));
+        return BC_OK;
+    }
+    CK(cudaMemsetAsync(d_bc, 0, sizeof(double) * (size_t)g->n, st));
+    CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
+    CK(cudaMemsetAsync(g->stats, 0, sizeof(DevStats), st));
+    g->last_inflight = 0;
+    g->launches = g->bc_launches = 0;
+    g->tev_used[0] = g->tev_used[1] = 0;
+    KParams p = base_params(g, d_bc);
+    p.sources = d_sources;
+    int rc = BC_OK;
+    const int strat = g->opt.strategy;
+    if (strat == BC_STRATEGY_SAMPLING) {
+        // Alg. 5: first n_samps sources WE, record max depth, decide, then the rest.
+        const long long ks = std::min<long long>(k, g->opt.n_samps);
+        KParams ps = p;
+        ps.launch_mode = LM_WE;
+        ps.src_base = 0;
+        ps.k = ks;
+        ps.keys = g->keys;
+        ps.work_counter = g->counters;
+        if (ks > 0) {
+            CK(cudaEventRecord(g->tev[0], st));
+            if ((rc = launch(g, ps, st))) return rc;
+            CK(cudaEventRecord(g->tev[1], st));
+            g->tev_used[0] = 1;
+        }
+        if (ks > 0) {
+            int P = 1;
+            while (P < ks) P <<= 1;
+            const double thresh = g->opt.gamma * std::log2((double)std::max(g->n, 1));
+            sampling_decide_kernel<<<1, 1024, sizeof(int) * (size_t)P, st>>>(g->keys, (int)ks, thresh,
+                                                                           g->flag, g->stats);
+            CK(cudaGetLastError());
+            g->launches++;
+            g->sampling_ran = 1;
+        }
+        KParams pm = p;
+        pm.launch_mode = LM_SAMPLED;
+        pm.src_base = ks;
+        pm.k = k - ks;
+        pm.work_counter = g->counters + 1;
+        if (pm.k > 0) {
+            CK(cudaEventRecord(g->tev[2], st));
+            if ((rc = launch(g, pm, st))) return rc;
+            CK(cudaEventRecord(g->tev[3], st));
+            g->tev_used[1] = 1;
+        }
+    } else {
+        KParams pm = p;
+        pm.launch_mode = strat == BC_STRATEGY_WE ? LM_WE : strat == BC_STRATEGY_EP ? LM_EP : LM_HYBRID;
+        pm.src_base = 0;
+        pm.k = k;
+        pm.work_counter = g->counters + 1;
+        if (pm.k > 0) {
+            CK(cudaEventRecord(g->tev[2], st));
+            if ((rc = launch(g, pm, st))) return rc;
+            CK(cudaEventRecord(g->tev[3], st));
+            g->tev_used[1] = 1;
+        }
+    }
+    if (!g->directed && g->n > 0) {
+        scale_kernel<<<std::min((g->n + 255) / 256, 148 * 8), 256, 0, st>>>(d_bc, g->n, 0.5);
+        CK(cudaGetLastError());
+        g->launches++;
+    }
+    CK(cudaEventRecord(g->done, st));
+    return BC_OK;
+}
+
+extern "C" int bc_compute_device(bc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc,
+                                 void *cuda_stream) {
+    if (!g || !d_bc) return fail(BC_EINVAL, "NULL argument");
+    if (!d_sources) k = g->n;
+    if (k < 0) return fail(BC_EINVAL, "k < 0");
+    DeviceGuard dg(g->device);
+    int rc = enqueue_compute(g, d_sources, k, d_bc, (cudaStream_t)cuda_stream);
+    if (rc == BC_OK) g_err[0] = 0;
+    return rc;
+}
+
+extern "C" int bc_compute(bc_graph *g, const int32_t *sources, int64_t num_sources, double *bc) {
+    if (!g || !bc) return fail(BC_EINVAL, "NULL argument");
+    long long k = sources ? num_sources : g->n;
+    if (k < 0) return fail(BC_EINVAL, "num_sources < 0");
+    if (sources)
+        for (long long i = 0; i < k; ++i)
+            if (sources[i] < 0 || sources[i] >= g->n)
+                return fail(BC_EINVAL, "sources[%lld]=%d out of range", i, sources[i]);
+    DeviceGuard dg(g->device);
+    CK(cudaEventSynchronize(g->done));
+    if (sources && k > g->src_cap) {
+        cudaFree(g->src_buf);
+        g->src_buf = nullptr;
+        g->src_cap = 0;
+        CK(cudaMalloc(&g->src_buf, sizeof(int) * (size_t)k));
+        g->src_cap = k;
+    }
+    if (!g->bc_buf) CK(cudaMalloc(&g->bc_buf, sizeof(double) * (size_t)std::max(g->n, 1)));
+    if (sources && k > 0)
+        CK(cudaMemcpyAsync(g->src_buf, sources, sizeof(int) * (size_t)k, cudaMemcpyHostToDevice, g->stream));
+    int rc = enqueue_compute(g, sources ? g->src_buf : nullptr, k, g->bc_buf, g->stream);
+    if (rc) return rc;
+    if (g->n > 0)
+        CK(cudaMemcpyAsync(bc, g->bc_buf, sizeof(double) * (size_t)g->n, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+    g_err[0] = 0;
+    return BC_OK;
+}
+
+extern "C" int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigma, double *delta,
+                                uint8_t *level_modes, int32_t max_levels, int32_t *num_levels) {
+    if (!g) return fail(BC_EINVAL, "NULL graph");
+    if (s < 0 || s >= g->n) return fail(BC_EINVAL, "source %d out of range", s);
+    if (level_modes && max_levels < 0) return fail(BC_EINVAL, "max_levels < 0");
+    DeviceGuard dg(g->device);
+    CK(cudaEventSynchronize(g->done));
+    const size_t n = (size_t)g->n;
+    const int ml = level_modes ? max_levels : 0;
+    int *dd = nullptr, *dn = nullptr, *dsrc = nullptr;
+    double *ds = nullptr, *ddel = nullptr, *dbc = nullptr;
+    unsigned char *dm = nullptr;
+    int rc = BC_OK;
+    cudaError_t e = cudaSuccess;
+    e = cudaMalloc(&dd, n * sizeof(int));
+    if (e == cudaSuccess) e = cudaMalloc(&ds, n * sizeof(double));
+    if (e == cudaSuccess) e = cudaMalloc(&ddel, n * sizeof(double));
+    if (e == cudaSuccess) e = cudaMalloc(&dbc, n * sizeof(double));
+    if (e == cudaSuccess) e = cudaMalloc(&dm, (size_t)std::max(ml, 1));
+    if (e == cudaSuccess) e = cudaMalloc(&dn, sizeof(int));
+    if (e == cudaSuccess) e = cudaMalloc(&dsrc, sizeof(int));
+    if (e == cudaSuccess) e = cudaMemsetAsync(dd, 0xFF, n * sizeof(int), g->stream);  // -1
+    if (e == cudaSuccess) e = cudaMemsetAsync(ds, 0, n * sizeof(double), g->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(ddel, 0, n * sizeof(double), g->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(dbc, 0, n * sizeof(double), g->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(dn, 0, sizeof(int), g->stream);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(dsrc, &s, sizeof(int), cudaMemcpyHostToDevice, g->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), g->stream);
+    DevStats *dst = nullptr;
+    if (e == cudaSuccess) e = cudaMalloc(&dst, sizeof(DevStats));
+    if (e == cudaSuccess) e = cudaMemsetAsync(dst, 0, sizeof(DevStats), g->stream);
+    if (e != cudaSuccess) rc = fail(e == cudaErrorMemoryAllocation ? BC_ENOMEM : BC_ECUDA, "%s", cudaGetErrorString(e));
+    if (rc == BC_OK) {
+        KParams p = base_params(g, dbc);
+        const int strat = g->opt.strategy;
+        p.launch_mode = strat == BC_STRATEGY_WE ? LM_WE : strat == BC_STRATEGY_EP ? LM_EP
+                      : strat == BC_STRATEGY_HYBRID ? LM_HYBRID : LM_SAMPLED;
+        p.sources = dsrc;
+        p.src_base = 0;
+        p.k = 1;
+        p.work_counter = g->counters;
+        p.dbg_d = dd;
+        p.dbg_sigma = ds;
+        p.dbg_delta = ddel;
+        p.dbg_modes = dm;
+        p.dbg_max_levels = ml;
+        p.dbg_nlevels = dn;
+        p.stats = dst;  // keep the last compute call's stats intact
+        rc = launch(g, p, g->stream);
+    }
+    int nl = 0;
+    if (rc == BC_OK) {
+        e = cudaStreamSynchronize(g->stream);
+        if (e == cudaSuccess && d) e = cudaMemcpy(d, dd, n * sizeof(int), cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess && sigma) e = cudaMemcpy(sigma, ds, n * sizeof(double), cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess && delta) e = cudaMemcpy(delta, ddel, n * sizeof(double), cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess) e = cudaMemcpy(&nl, dn, sizeof(int), cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess && level_modes && ml > 0)
+            e = cudaMemcpy(level_modes, dm, (size_t)std::min(ml, nl), cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) rc = fail(BC_ECUDA, "%s", cudaGetErrorString(e));
+    }
+    if (rc == BC_OK && num_levels) *num_levels = nl;
+    cudaFree(dd);
+    cudaFree(ds);
+    cudaFree(ddel);
+    cudaFree(dbc);
+    cudaFree(dm);
+    cudaFree(dn);
+    cudaFree(dsrc);
+    cudaFree(dst);
+    if (rc == BC_OK) g_err[0] = 0;
+    return rc;
+}
+
+extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {
+    if (!g || !st) return fail(BC_EINVAL, "NULL argument");
+    DeviceGuard dg(g->device);
+    CK(cudaEventSynchronize(g->done));
+    CK(cudaStreamSynchronize(g->stream));
+    DevStats h;
+    CK(cudaMemcpy(&h, g->stats, sizeof(h), cudaMemcpyDeviceToHost));
+    st->sources = (int64_t)h.sources;
+    st->levels = (int64_t)h.levels;
+    st->we_levels = (int64_t)h.we_levels;
+    st->ep_levels = (int64_t)h.ep_levels;
+    st->n_reached = (int64_t)h.n_reached;
+    st->arcs_reached = (int64_t)h.arcs_reached;
+    st->dag_arcs = (int64_t)h.dag_arcs;
+    st->arcs_scanned = (int64_t)h.arcs_scanned;
+    const int samp = g->opt.strategy == BC_STRATEGY_SAMPLING && g->sampling_ran;
+    st->sampling_ep = samp ? h.sampling_ep : -1;
+    st->sampling_median = samp ? h.sampling_median : -1;
+    st->sigma_inexact = h.sigma_inexact;
+    st->inflight = g->last_inflight;
+    st->kernel_launches = g->launches;
+    st->bc_kernel_launches = g->bc_launches;
+    st->kernel_ms = 0.0;
+    for (int i = 0; i < 2; ++i)
+        if (g->tev_used[i]) {
+            float ms = 0.f;
+            CK(cudaEventElapsedTime(&ms, g->tev[2 * i], g->tev[2 * i + 1]));
+            st->kernel_ms += ms;
+        }
+    return BC_OK;
+}
