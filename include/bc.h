@@ -71,6 +71,12 @@ typedef struct bc_options {
     int32_t inflight;        /* sources processed concurrently (one CTA each); 0 = auto        */
     int32_t backward_we;     /* 1: backward always WE (Alg. 3); 0 (default): backward level L
                                 uses the mode forward level L used (R8)              */
+    /* Implementation knobs (do not change results beyond fp64 rounding order): */
+    int32_t block_threads;   /* threads per CTA: 0 = auto, 256 or 512                           */
+    int32_t seq_max_deg;     /* rows up to this degree are summed by one thread in CSR order;
+                                longer rows CTA-cooperatively.  0 = auto (32)                  */
+    int32_t level_store;     /* 0 = auto, 1 = exact int32 d in HBM, 2 = 2-bit codes in shared
+                                memory (undirected graphs whose codes fit; else EINVAL)        */
 } bc_options;
 
 typedef struct bc_stats {

@@ -29,7 +29,8 @@ class bc_options(ctypes.Structure):
     _fields_ = [("strategy", ctypes.c_int32), ("alpha", ctypes.c_int32), ("beta", ctypes.c_int32),
                 ("gamma", ctypes.c_double), ("n_samps", ctypes.c_int32),
                 ("ep_min_frontier", ctypes.c_int32), ("inflight", ctypes.c_int32),
-                ("backward_we", ctypes.c_int32)]
+                ("backward_we", ctypes.c_int32), ("block_threads", ctypes.c_int32),
+                ("seq_max_deg", ctypes.c_int32), ("level_store", ctypes.c_int32)]
 
 
 class bc_stats(ctypes.Structure):

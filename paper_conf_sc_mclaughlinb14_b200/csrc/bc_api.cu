@@ -58,7 +58,16 @@ struct bc_graph {
     int nnz = 0;
     int directed = 0;
     int num_sms = 0;
-    int occ_slots = 0;  // occupancy-limited CTA count
+    // kernel configuration (see configure()): one without / one with the EP bitmap
+    struct KCfg {
+        const void *fn = nullptr;
+        int nt = 256;
+        size_t dyn = 0;   // dynamic shared memory bytes
+        int per_sm = 1;   // resident CTAs per SM
+    } cfg_we, cfg_ep;
+    int use_smem = 0;     // 2-bit level codes in shared memory
+    int code_words = 0, fb_words = 0;
+    int seq_max_deg = 32;
     // graph
     int *ro = nullptr, *col = nullptr, *src = nullptr;
     int *iro = nullptr, *icol = nullptr, *isrc = nullptr;
@@ -98,6 +107,9 @@ extern "C" void bc_default_options(bc_options *o) {
     o->ep_min_frontier = 512;
     o->inflight = 0;
     o->backward_we = 0;
+    o->block_threads = 0;
+    o->seq_max_deg = 0;
+    o->level_store = 0;
 }
 
 extern "C" const char *bc_last_error(void) { return g_err; }
@@ -117,8 +129,48 @@ static void free_workspace(bc_graph *g) {
 }
 
 static size_t slot_bytes(const bc_graph *g) {
-    return g->stride_n * (sizeof(int) + 2 * sizeof(double) + sizeof(int)) +
+    return g->stride_n * ((g->use_smem ? 0 : sizeof(int)) + 2 * sizeof(double) + sizeof(int)) +
            g->stride_e * (sizeof(int) + 1);
+}
+
+template <bool DIR, class LV>
+static const void *kernel_for(int nt) {
+    return nt == 512 ? (const void *)bc_kernel<DIR, LV, 512> : (const void *)bc_kernel<DIR, LV, 256>;
+}
+
+// Choose level store, block size and shared memory for both launch kinds
+// (with / without the EP frontier bitmap) and their occupancy.
+static int configure(bc_graph *g) {
+    const bc_options &o = g->opt;
+    const size_t code_bytes = (((size_t)g->n + 15) / 16) * 4;
+    const size_t fb_bytes = (((size_t)g->n + 31) / 32) * 4;
+    const size_t smem_cap = 200 * 1024;  // leaves room for the static part (< 16 KB)
+    const bool fits = !g->directed && code_bytes + fb_bytes <= smem_cap;
+    if (o.level_store == 2 && !fits)
+        return fail(BC_EINVAL, "level_store=2 needs an undirected graph with n <= ~%zu", smem_cap * 8 / 3);
+    g->use_smem = o.level_store == 1 ? 0 : (fits ? 1 : 0);
+    int nt = o.block_threads;
+    if (nt == 0) nt = 256;
+    if (nt != 256 && nt != 512) return fail(BC_EINVAL, "block_threads must be 0, 256 or 512");
+    g->seq_max_deg = o.seq_max_deg > 0 ? o.seq_max_deg : 32;
+    g->code_words = g->use_smem ? (int)(code_bytes / 4) : 0;
+    g->fb_words = g->use_smem ? (int)(fb_bytes / 4) : 0;
+    const void *fn;
+    if (g->directed) fn = kernel_for<true, GlobalLevels>(nt);
+    else if (g->use_smem) fn = kernel_for<false, SmemCodes>(nt);
+    else fn = kernel_for<false, GlobalLevels>(nt);
+    g->cfg_we.fn = g->cfg_ep.fn = fn;
+    g->cfg_we.nt = g->cfg_ep.nt = nt;
+    g->cfg_we.dyn = g->use_smem ? code_bytes : 0;
+    g->cfg_ep.dyn = g->use_smem ? code_bytes + fb_bytes : 0;
+    CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_ep.dyn));
+    for (auto *c : {&g->cfg_we, &g->cfg_ep}) {
+        int per_sm = 0;
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, c->fn, c->nt, c->dyn));
+        if (per_sm < 1) return fail(BC_EINTERNAL, "kernel cannot be resident (dyn smem %zu)", c->dyn);
+        c->per_sm = per_sm;
+    }
+    return BC_OK;
 }
 
 static int alloc_workspace(bc_graph *g) {
@@ -126,7 +178,8 @@ static int alloc_workspace(bc_graph *g) {
     g->stride_n = (size_t)std::max(g->n, 1);
     g->stride_n = (g->stride_n + 31) & ~(size_t)31;  // 128-byte aligned slots
     g->stride_e = g->stride_n + 32;
-    int want = g->opt.inflight > 0 ? std::min(g->opt.inflight, g->occ_slots) : g->occ_slots;
+    const int occ = std::max(g->cfg_we.per_sm, g->cfg_ep.per_sm) * g->num_sms;
+    int want = g->opt.inflight > 0 ? std::min(g->opt.inflight, occ) : occ;
     size_t free_b = 0, total_b = 0;
     CK(cudaMemGetInfo(&free_b, &total_b));
     size_t per = slot_bytes(g);
@@ -134,13 +187,13 @@ static int alloc_workspace(bc_graph *g) {
     int cap = (int)std::max<size_t>(1, budget / std::max<size_t>(per, 1));
     g->slots = std::max(1, std::min(want, cap));
     size_t ns = (size_t)g->slots;
-    CK(cudaMalloc(&g->d, ns * g->stride_n * sizeof(int)));
+    if (!g->use_smem) CK(cudaMalloc(&g->d, ns * g->stride_n * sizeof(int)));
     CK(cudaMalloc(&g->sigma, ns * g->stride_n * sizeof(double)));
     CK(cudaMalloc(&g->omega, ns * g->stride_n * sizeof(double)));
     CK(cudaMalloc(&g->S, ns * g->stride_n * sizeof(int)));
     CK(cudaMalloc(&g->ends, ns * g->stride_e * sizeof(int)));
     CK(cudaMalloc(&g->modes, ns * g->stride_e));
-    CK(cudaMemset(g->d, 0x7F, ns * g->stride_n * sizeof(int)));  // INF = 0x7F7F7F7F
+    if (!g->use_smem) CK(cudaMemset(g->d, 0x7F, ns * g->stride_n * sizeof(int)));  // INF = 0x7F7F7F7F
     CK(cudaMemset(g->sigma, 0, ns * g->stride_n * sizeof(double)));
     CK(cudaMemset(g->omega, 0, ns * g->stride_n * sizeof(double)));
     CK(cudaDeviceSynchronize());
@@ -213,12 +266,10 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col) {
     CK(cudaMalloc(&g->stats, sizeof(DevStats)));
     CK(cudaMemset(g->stats, 0, sizeof(DevStats)));
     CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
-    int per_sm = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-        &per_sm, g->directed ? (const void *)bc_kernel<true> : (const void *)bc_kernel<false>, NT, 0));
-    g->occ_slots = std::max(1, per_sm) * g->num_sms;
     bc_default_options(&g->opt);
-    int rc = alloc_workspace(g);
+    int rc = configure(g);
+    if (rc) return rc;
+    rc = alloc_workspace(g);
     if (rc) return rc;
     CK(cudaDeviceSynchronize());
     return BC_OK;
@@ -267,13 +318,29 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     if (!g || !o) return fail(BC_EINVAL, "NULL argument");
     if (o->strategy < 0 || o->strategy > 3) return fail(BC_EINVAL, "bad strategy %d", o->strategy);
     if (o->n_samps < 1 || o->n_samps > 8192) return fail(BC_EINVAL, "n_samps must be in [1, 8192]");
-    if (o->alpha < 0 || o->beta < 0 || o->ep_min_frontier < 0 || o->inflight < 0 || !(o->gamma >= 0))
-        return fail(BC_EINVAL, "negative parameter");
+    if (o->alpha < 0 || o->beta < 0 || o->ep_min_frontier < 0 || o->inflight < 0 || !(o->gamma >= 0) ||
+        o->seq_max_deg < 0 || o->level_store < 0 || o->level_store > 2)
+        return fail(BC_EINVAL, "invalid parameter");
+    if (o->block_threads != 0 && o->block_threads != 256 && o->block_threads != 512)
+        return fail(BC_EINVAL, "block_threads must be 0, 256 or 512");
     DeviceGuard dg(g->device);
     if (g->done) CK(cudaEventSynchronize(g->done));
-    const int realloc = o->inflight != g->opt.inflight;
+    const bc_options old = g->opt;
     g->opt = *o;
-    if (realloc) return alloc_workspace(g);
+    int rc = configure(g);
+    if (rc) {
+        g->opt = old;
+        configure(g);
+        return rc;
+    }
+    const int old_slots = g->slots;
+    const int realloc = o->inflight != old.inflight || o->level_store != old.level_store ||
+                        o->block_threads != old.block_threads;
+    if (realloc) {
+        rc = alloc_workspace(g);
+        if (rc) return rc;
+    }
+    (void)old_slots;
     return BC_OK;
 }
 
@@ -307,16 +374,23 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     p.beta = g->opt.beta;
     p.ep_min_frontier = g->opt.ep_min_frontier;
     p.backward_we = g->opt.backward_we;
+    p.code_words = g->code_words;
+    p.seq_max_deg = g->seq_max_deg;
     p.stats = g->stats;
     p.sampled_flag = g->flag;
     return p;
 }
 
-static int launch(bc_graph *g, const KParams &p, cudaStream_t st) {
-    if (p.k <= 0) return BC_OK;
-    int grid = (int)std::min<long long>(g->slots, p.k);
-    if (g->directed) bc_kernel<true><<<grid, NT, 0, st>>>(p);
-    else bc_kernel<false><<<grid, NT, 0, st>>>(p);
+static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
+    if (p0.k <= 0) return BC_OK;
+    KParams p = p0;
+    const bool ep_possible = p.launch_mode != LM_WE;
+    const bc_graph::KCfg &c = ep_possible ? g->cfg_ep : g->cfg_we;
+    p.fb_words = ep_possible ? g->fb_words : 0;
+    const long long cap = std::min<long long>(g->slots, (long long)c.per_sm * g->num_sms);
+    const int grid = (int)std::min<long long>(cap, p.k);
+    void *args[] = {&p};
+    CK(cudaLaunchKernel(c.fn, dim3(grid), dim3(c.nt), args, c.dyn, st));
     g->last_inflight = std::max(g->last_inflight, grid);
     g->launches++;
     g->bc_launches++;

@@ -3,19 +3,27 @@
 // One CTA owns one source at a time ("coarse-grained" root parallelism, P:118,
 // P:198) and loops: Alg. 1 init -> forward levels (Alg. 2) in WE or
 // EP mode -> backward levels (Alg. 3) -> BC update (Eq. 3) ->
-// reset of only the touched vertices.  Sources are pulled from a global atomic
-// counter so the grid is persistent (one CTA per workspace slot).
+// reset of the touched state.  Sources are pulled from a global atomic counter,
+// so the grid is persistent (one CTA per workspace slot).
 //
-// B200 choices (DESIGN.md §4):
+// B200 choices (DESIGN.md §8):
+//  * Level state policy.  Undirected graphs whose 2-bit level codes fit in shared
+//    memory keep d as a code per vertex in SMEM (0 = unvisited, 1 + L mod 3):
+//    every neighbour of a level-L vertex lies on L-1, L or L+1, so the code
+//    decides the predecessor / successor / unvisited tests exactly, and every
+//    probe of Alg. 2 l.5/l.7 and Alg. 3 l.7 is a shared-memory load instead of a
+//    random HBM sector.  Directed or large graphs keep exact int32 d in HBM.
 //  * sigma is PULLED (sigma[w] = sum of sigma over w's level-(L-1) neighbours)
 //    when w itself is expanded, fused with w's discovery scan: one CSR row read
-//    serves both, no sigma atomics in WE mode, and rows of degree <= SEQ_MAX_DEG
+//    serves both, no sigma atomics in WE mode, and rows of degree <= seq_max_deg
 //    are summed by one thread in CSR order = the oracle's order (bit-exact).
-//  * the queue is S itself: level L+1 is appended at S[ends[L+1]...], so Alg. 2's
-//    Q_next -> Q_curr copy (l.15-17) disappears (§8(a) a4).
-//  * rows of degree > SEQ_MAX_DEG are expanded CTA-cooperatively: block scan of
+//  * the queue is S itself: level L+1 is appended at S[ends[L+1]...] with a
+//    warp-aggregated atomic, so Alg. 2's Q_next -> Q_curr copy disappears.
+//  * rows of degree > seq_max_deg are expanded CTA-cooperatively: block scan of
 //    their degrees, arcs dealt round-robin to all threads, owner found by binary
 //    search in shared memory, warp-segmented reduction of the partial sums.
+//  * EP levels stream src[]/col[] with 16-byte vector loads and test frontier
+//    membership in a shared-memory bitmap.
 //  * backward uses omega[v] = (1 + delta[v]) / sigma[v]: one 8-byte gather per
 //    DAG arc, delta[w] = sigma[w] * sum(omega of successors).
 #pragma once
@@ -25,10 +33,7 @@
 
 namespace bcdev {
 
-constexpr int NT = 256;             // threads per CTA
-constexpr int NWARP = NT / 32;
-constexpr int SEQ_MAX_DEG = 32;     // rows up to this degree: one thread, CSR order
-constexpr int INF = 0x7F7F7F7F;     // "infinity" distance (memset-able byte pattern)
+constexpr int INF = 0x7F7F7F7F;  // "infinity" distance (memset-able byte pattern)
 constexpr unsigned FULL = 0xFFFFFFFFu;
 constexpr double TWO53 = 9007199254740992.0;
 
@@ -58,7 +63,7 @@ struct KParams {
     long long k;                      // sources in this launch
     unsigned long long *work_counter;
     // workspace (slot-major)
-    int *d;
+    int *d;                           // GlobalLevels only
     double *sigma;
     double *omega;
     int *S;
@@ -67,6 +72,10 @@ struct KParams {
     size_t stride_n;     // elements per slot for d/sigma/omega/S
     size_t stride_e;     // elements per slot for ends/modes
     double *bc;
+    // shared-memory level codes (SmemCodes): 32-bit words of codes / of the EP bitmap
+    int code_words;
+    int fb_words;        // 0: this launch never runs an EP level
+    int seq_max_deg;
     // strategy
     int launch_mode;
     const int *sampled_flag;  // LM_SAMPLED: 1 = EP run
@@ -83,22 +92,14 @@ struct KParams {
     int *dbg_nlevels;
 };
 
+template <int NT>
 struct Smem {
     long long idx;
     int s_len;
-    int warp_tot[NWARP + 1];
+    int warp_tot[NT / 32 + 1];
     int off[NT];
     int beg[NT];
     double acc[NT];
-};
-
-struct Slot {
-    int *d;
-    double *sigma;
-    double *omega;
-    int *S;
-    int *ends;
-    unsigned char *modes;
 };
 
 struct Counters {
@@ -106,9 +107,61 @@ struct Counters {
     int inexact = 0;
 };
 
+// ------------------------------------------------------------ level policies
+
+// Exact int32 distances in HBM (directed graphs, or graphs too large for SMEM codes).
+struct GlobalLevels {
+    static constexpr int UNVISITED = INF;
+    int *d;
+    uint32_t *fb;  // unused
+    __device__ __forceinline__ int probe(int u) const { return d[u]; }
+    __device__ __forceinline__ static int key(int L) { return L; }  // L = -1: matches nothing
+    __device__ __forceinline__ bool discover(int u, int L1) const {
+        return atomicCAS(&d[u], INF, L1) == INF;
+    }
+    __device__ __forceinline__ bool in_frontier(int x, int L) const { return d[x] == L; }
+    __device__ __forceinline__ void set_source(int s) const { d[s] = 0; }
+    __device__ __forceinline__ void reset_vertex(int v) const { d[v] = INF; }
+    template <int NT> __device__ __forceinline__ void reset_all(int) const {}
+    template <int NT> __device__ __forceinline__ void prepare_frontier(const int *, int, int, int) const {}
+};
+
+// 2-bit level codes in shared memory, undirected graphs only (see header).
+struct SmemCodes {
+    static constexpr int UNVISITED = 0;
+    uint32_t *w;   // codes, 16 vertices per word
+    uint32_t *fb;  // EP frontier bitmap, 32 vertices per word
+    __device__ __forceinline__ int probe(int u) const { return (w[u >> 4] >> ((u & 15) << 1)) & 3; }
+    __device__ __forceinline__ static int key(int L) { return L < 0 ? 4 : (L % 3) + 1; }
+    __device__ __forceinline__ bool discover(int u, int L1) const {
+        const uint32_t sh = (uint32_t)(u & 15) << 1;
+        const uint32_t old = atomicOr(&w[u >> 4], (uint32_t)key(L1) << sh);
+        return ((old >> sh) & 3u) == 0u;
+    }
+    __device__ __forceinline__ bool in_frontier(int x, int) const { return (fb[x >> 5] >> (x & 31)) & 1u; }
+    __device__ __forceinline__ void set_source(int s) const { w[s >> 4] |= (uint32_t)key(0) << ((s & 15) << 1); }
+    __device__ __forceinline__ void reset_vertex(int) const {}
+    template <int NT> __device__ __forceinline__ void reset_all(int words) const {
+        for (int i = threadIdx.x; i < words; i += NT) w[i] = 0u;
+    }
+    // Bitmap of S[lo, hi) (one EP level).  Ends with a barrier.
+    template <int NT>
+    __device__ __forceinline__ void prepare_frontier(const int *S, int lo, int hi, int words) const {
+        for (int i = threadIdx.x; i < words; i += NT) fb[i] = 0u;
+        __syncthreads();
+        for (int i = lo + threadIdx.x; i < hi; i += NT) {
+            const int v = S[i];
+            atomicOr(&fb[v >> 5], 1u << (v & 31));
+        }
+        __syncthreads();
+    }
+};
+
 // ------------------------------------------------------------------ helpers
 
-__device__ __forceinline__ int block_exclusive_scan(int x, int &total, Smem &sm) {
+template <int NT>
+__device__ __forceinline__ int block_exclusive_scan(int x, int &total, Smem<NT> &sm) {
+    constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     int incl = x;
 #pragma unroll
@@ -119,30 +172,34 @@ __device__ __forceinline__ int block_exclusive_scan(int x, int &total, Smem &sm)
     if (lane == 31) sm.warp_tot[wid] = incl;
     __syncthreads();
     if (wid == 0) {
-        int v = lane < NWARP ? sm.warp_tot[lane] : 0;
+        int v = lane < NW ? sm.warp_tot[lane] : 0;
         int inc = v;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             int y = __shfl_up_sync(FULL, inc, o);
             if (lane >= o) inc += y;
         }
-        if (lane < NWARP) sm.warp_tot[lane] = inc - v;
-        if (lane == NWARP - 1) sm.warp_tot[NWARP] = inc;
+        if (lane < NW) sm.warp_tot[lane] = inc - v;
+        if (lane == NW - 1) sm.warp_tot[NW] = inc;
     }
     __syncthreads();
-    total = sm.warp_tot[NWARP];
+    total = sm.warp_tot[NW];
     return incl - x + sm.warp_tot[wid];
 }
 
-__device__ __forceinline__ void discover(int *d, int *S, int *s_len, int u, int L1) {
-    if (atomicCAS(&d[u], INF, L1) == INF) {
-        int pos = atomicAdd(s_len, 1);
-        S[pos] = u;
-    }
+// Append u to S (Q_next) with one shared atomic per group of converged lanes.
+__device__ __forceinline__ void enqueue(int *S, int *s_len, int u) {
+    const unsigned m = __activemask();
+    const int lane = threadIdx.x & 31;
+    const int leader = __ffs(m) - 1;
+    int base = 0;
+    if (lane == leader) base = atomicAdd(s_len, __popc(m));
+    base = __shfl_sync(m, base, leader);
+    S[base + __popc(m & ((1u << lane) - 1u))] = u;
 }
 
-// Segmented (by non-decreasing owner) warp sum; returns true for the tail lane of
-// each segment, which then holds the segment total in `val`.
+// Segmented (by non-decreasing owner) warp sum; true for the tail lane of each
+// segment, which then holds the segment total in `val`.
 __device__ __forceinline__ bool warp_segmented_sum(int owner, double &val) {
     const int lane = threadIdx.x & 31;
 #pragma unroll
@@ -155,15 +212,16 @@ __device__ __forceinline__ bool warp_segmented_sum(int owner, double &val) {
     return owner >= 0 && (lane == 31 || nxt != owner);
 }
 
-// Generic "row pass" over a contiguous range of S: every vertex v = S[i] has its
-// row [rows[v], rows[v+1]) of `cols` inspected; op(u) returns a double
-// contribution.  Returns (for the calling thread) the sum for the vertex it owns in
-// the CURRENT tile through `body` -- the pass calls finish(v, acc) once per vertex.
-template <class Probe, class Op, class Finish>
+// Row pass over the vertices S[lo, hi): every row [rows[v], rows[v+1]) of `cols`
+// is inspected; op(u, probe(u)) returns a double contribution; finish(v, sum, big)
+// is called once per vertex.  Rows of degree <= seq_max are summed by their owner
+// thread in CSR order; longer rows by the whole CTA (load-balanced).
+template <int NT, class Probe, class Op, class Finish>
 __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int hi,
                                          const int *__restrict__ rows,
-                                         const int *__restrict__ cols, Smem &sm,
-                                         Counters &c, Probe probe, Op op, Finish finish) {
+                                         const int *__restrict__ cols, int seq_max,
+                                         Smem<NT> &sm, Counters &c, Probe probe, Op op,
+                                         Finish finish) {
     for (int base = lo; base < hi; base += NT) {
         const int i = base + threadIdx.x;
         int v = -1, beg = 0, deg = 0;
@@ -173,10 +231,9 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             deg = rows[v + 1] - beg;
         }
         c.scanned += deg;
-        const bool big = deg > SEQ_MAX_DEG;
+        const bool big = deg > seq_max;
         double acc = 0.0;
         if (v >= 0 && !big) {
-            // one thread, CSR order (same summation order as the oracle)
             int a = beg;
             const int e = beg + deg;
             for (; a + 4 <= e; a += 4) {
@@ -193,7 +250,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             }
         }
         int total;
-        const int off = block_exclusive_scan(big ? deg : 0, total, sm);
+        const int off = block_exclusive_scan<NT>(big ? deg : 0, total, sm);
         if (total > 0) {  // block-uniform
             sm.off[threadIdx.x] = off;
             sm.beg[threadIdx.x] = beg;
@@ -205,8 +262,9 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
                 double val = 0.0;
                 if (j < total) {
                     int lo2 = 0, hi2 = NT - 1;  // last t with off[t] <= j
+#pragma unroll 1
                     while (lo2 < hi2) {
-                        int mid = (lo2 + hi2 + 1) >> 1;
+                        const int mid = (lo2 + hi2 + 1) >> 1;
                         if (sm.off[mid] <= j) lo2 = mid; else hi2 = mid - 1;
                     }
                     owner = lo2;
@@ -228,7 +286,7 @@ __device__ __forceinline__ int next_mode(const KParams &p, int mode, int run_ep,
     case LM_WE: return MODE_WE;
     case LM_EP: return MODE_EP;
     case LM_HYBRID: {  // Alg. 4
-        int change = q_next > q_curr ? q_next - q_curr : q_curr - q_next;
+        const int change = q_next > q_curr ? q_next - q_curr : q_curr - q_next;
         if (change > p.alpha) return q_next > p.beta ? MODE_EP : MODE_WE;
         return mode;
     }
@@ -239,19 +297,17 @@ __device__ __forceinline__ int next_mode(const KParams &p, int mode, int run_ep,
 
 // ------------------------------------------------------------------ forward
 
-template <bool DIR>
-__device__ void forward_we(const KParams &p, const Slot &sl, int L, int lo, int hi, Smem &sm,
-                           Counters &c) {
-    int *d = sl.d;
-    double *sigma = sl.sigma;
-    int *S = sl.S;
-    const int L1 = L + 1, Lm1 = L - 1;
+template <bool DIR, int NT, class LV>
+__device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S, int L, int lo,
+                           int hi, Smem<NT> &sm, Counters &c) {
+    const int L1 = L + 1;
+    const int kprev = LV::key(L - 1);
+    auto probe = [&](int u) -> int { return lv.probe(u); };
     if (!DIR) {
         // fused: discovery of level L+1 and sigma pull for level L in one row scan
-        auto probe = [&](int u) -> int { return d[u]; };
-        auto op = [&](int u, int du) -> double {
-            if (du == Lm1) { c.dag++; return sigma[u]; }
-            if (du == INF) discover(d, S, &sm.s_len, u, L1);
+        auto op = [&](int u, int k) -> double {
+            if (k == kprev) { c.dag++; return sigma[u]; }
+            if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S, &sm.s_len, u);
             return 0.0;
         };
         auto fin = [&](int v, double acc, bool big) {
@@ -261,134 +317,168 @@ __device__ void forward_we(const KParams &p, const Slot &sl, int L, int lo, int 
             }
         };
         const unsigned long long before = c.scanned;
-        row_pass(S, lo, hi, p.ro, p.col, sm, c, probe, op, fin);
+        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, sm, c, probe, op, fin);
         c.arcs_reached += c.scanned - before;
     } else {
-        auto probe = [&](int u) -> int { return d[u]; };
-        auto op1 = [&](int u, int du) -> double {
-            if (du == INF) discover(d, S, &sm.s_len, u, L1);
+        auto op1 = [&](int u, int k) -> double {
+            if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S, &sm.s_len, u);
             return 0.0;
         };
         auto fin1 = [&](int, double, bool) {};
         const unsigned long long before = c.scanned;
-        row_pass(S, lo, hi, p.ro, p.col, sm, c, probe, op1, fin1);
+        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, sm, c, probe, op1, fin1);
         c.arcs_reached += c.scanned - before;
         if (L > 0) {
-            auto op2 = [&](int u, int du) -> double {
-                if (du == Lm1) { c.dag++; return sigma[u]; }
+            auto op2 = [&](int u, int k) -> double {
+                if (k == kprev) { c.dag++; return sigma[u]; }
                 return 0.0;
             };
             auto fin2 = [&](int v, double acc, bool big) {
                 sigma[v] = acc;
                 if (big && acc >= TWO53) c.inexact = 1;
             };
-            row_pass(S, lo, hi, p.iro, p.icol, sm, c, probe, op2, fin2);
+            row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, sm, c, probe, op2, fin2);
         }
     }
 }
 
-template <bool DIR>
-__device__ void forward_ep(const KParams &p, const Slot &sl, int L, int lo, int hi, Smem &sm,
-                           Counters &c) {
-    int *d = sl.d;
-    double *sigma = sl.sigma;
-    int *S = sl.S;
-    const int L1 = L + 1, Lm1 = L - 1;
-    // Sum of degrees of the frontier (for the TEPS byte model only).
-    for (int i = lo + threadIdx.x; i < hi; i += NT) {
-        int v = S[i];
+// Thread-per-arc scan of ALL arcs (a_src[i] -> a_dst[i]) restricted to sources in
+// the current frontier (Jia et al. EP): 16-byte loads of src[], col[]
+// loaded only when one of the four arcs starts in the frontier.
+template <int NT, class LV, class Arc>
+__device__ __forceinline__ void ep_scan(const int *__restrict__ a_src, const int *__restrict__ a_dst,
+                                        int nnz, const LV &lv, int L, Arc arc) {
+    const int n4 = nnz >> 2;
+    const int4 *s4 = reinterpret_cast<const int4 *>(a_src);
+    const int4 *d4 = reinterpret_cast<const int4 *>(a_dst);
+#pragma unroll 2
+    for (int q = threadIdx.x; q < n4; q += NT) {
+        const int4 xs = s4[q];
+        const bool f0 = lv.in_frontier(xs.x, L), f1 = lv.in_frontier(xs.y, L);
+        const bool f2 = lv.in_frontier(xs.z, L), f3 = lv.in_frontier(xs.w, L);
+        if (f0 | f1 | f2 | f3) {
+            const int4 ys = d4[q];
+            if (f0) arc(xs.x, ys.x);
+            if (f1) arc(xs.y, ys.y);
+            if (f2) arc(xs.z, ys.z);
+            if (f3) arc(xs.w, ys.w);
+        }
+    }
+    for (int a = (n4 << 2) + threadIdx.x; a < nnz; a += NT) {
+        const int x = a_src[a];
+        if (lv.in_frontier(x, L)) arc(x, a_dst[a]);
+    }
+}
+
+template <bool DIR, int NT, class LV>
+__device__ void forward_ep(const KParams &p, const LV &lv, double *sigma, int *S, int L, int lo,
+                           int hi, Smem<NT> &sm, Counters &c) {
+    const int L1 = L + 1;
+    const int kprev = LV::key(L - 1);
+    lv.template prepare_frontier<NT>(S, lo, hi, p.fb_words);
+    for (int i = lo + threadIdx.x; i < hi; i += NT) {  // sum of frontier degrees (byte model)
+        const int v = S[i];
         c.arcs_reached += (unsigned long long)(p.ro[v + 1] - p.ro[v]);
     }
-    // Thread per arc over ALL arcs (Jia et al. EP).
-    for (int a = threadIdx.x; a < p.nnz; a += NT) {
-        int x = p.src[a];
-        if (d[x] != L) continue;
-        int y = p.col[a];
-        int dy = d[y];
-        if (dy == INF) {
-            discover(d, S, &sm.s_len, y, L1);
-        } else if (!DIR && dy == Lm1) {
-            double s = sigma[y];
-            double old = atomicAdd(&sigma[x], s);
+    auto arc = [&](int x, int y) {
+        const int k = lv.probe(y);
+        if (k == LV::UNVISITED) {
+            if (lv.discover(y, L1)) enqueue(S, &sm.s_len, y);
+        } else if (!DIR && k == kprev) {
+            const double s = sigma[y];
+            const double old = atomicAdd(&sigma[x], s);
             c.dag++;
             if (old + s >= TWO53) c.inexact = 1;
         }
-    }
-    c.scanned += (unsigned long long)p.nnz;
+    };
+    ep_scan<NT>(p.src, p.col, p.nnz, lv, L, arc);
+    if (threadIdx.x == 0) c.scanned += (unsigned long long)p.nnz;
     if (DIR && L > 0) {
-        for (int a = threadIdx.x; a < p.nnz; a += NT) {
-            int x = p.isrc[a];
-            if (d[x] != L) continue;
-            int y = p.icol[a];
-            if (d[y] == Lm1) {
-                double s = sigma[y];
-                double old = atomicAdd(&sigma[x], s);
+        auto arc_in = [&](int x, int y) {
+            if (lv.probe(y) == kprev) {
+                const double s = sigma[y];
+                const double old = atomicAdd(&sigma[x], s);
                 c.dag++;
                 if (old + s >= TWO53) c.inexact = 1;
             }
-        }
-        c.scanned += (unsigned long long)p.nnz;
+        };
+        ep_scan<NT>(p.isrc, p.icol, p.nnz, lv, L, arc_in);
+        if (threadIdx.x == 0) c.scanned += (unsigned long long)p.nnz;
     }
 }
 
 // ------------------------------------------------------------------ backward
 
-__device__ __forceinline__ void finish_dependency(const KParams &p, const Slot &sl, int w,
-                                                  double acc) {
-    const double sw = sl.sigma[w];
+__device__ __forceinline__ void finish_dependency(const KParams &p, const double *sigma,
+                                                  double *omega, int w, double acc) {
+    const double sw = sigma[w];
     const double delta = sw * acc;                 // delta[w] = sum sw/sigma[v] (1+delta[v])
-    sl.omega[w] = (1.0 + delta) / sw;
+    omega[w] = (1.0 + delta) / sw;
     if (delta != 0.0) atomicAdd(&p.bc[w], delta);  // Eq. 3
     if (p.dbg_delta) p.dbg_delta[w] = delta;
 }
 
-__device__ void backward_we(const KParams &p, const Slot &sl, int L, int lo, int hi, Smem &sm,
-                            Counters &c) {
-    const int *d = sl.d;
-    const double *omega = sl.omega;
-    const int L1 = L + 1;
-    auto probe = [&](int v) -> int { return d[v]; };
-    auto op = [&](int v, int dv) -> double { return dv == L1 ? omega[v] : 0.0; };
-    auto fin = [&](int w, double acc, bool) { finish_dependency(p, sl, w, acc); };
-    row_pass(sl.S, lo, hi, p.ro, p.col, sm, c, probe, op, fin);
+template <int NT, class LV>
+__device__ void backward_we(const KParams &p, const LV &lv, const double *sigma, double *omega,
+                            const int *S, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
+    const int knext = LV::key(L + 1);
+    auto probe = [&](int v) -> int { return lv.probe(v); };
+    auto op = [&](int v, int k) -> double { return k == knext ? omega[v] : 0.0; };
+    auto fin = [&](int w, double acc, bool) { finish_dependency(p, sigma, omega, w, acc); };
+    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, sm, c, probe, op, fin);
 }
 
-__device__ void backward_ep(const KParams &p, const Slot &sl, int L, int lo, int hi, Smem &sm,
-                            Counters &c) {
-    const int *d = sl.d;
-    double *omega = sl.omega;
-    const int L1 = L + 1;
-    for (int a = threadIdx.x; a < p.nnz; a += NT) {
-        int x = p.src[a];
-        if (d[x] != L) continue;
-        int y = p.col[a];
-        if (d[y] == L1) atomicAdd(&omega[x], omega[y]);  // omega[x] == 0 until finished
-    }
-    c.scanned += (unsigned long long)p.nnz;
+template <int NT, class LV>
+__device__ void backward_ep(const KParams &p, const LV &lv, const double *sigma, double *omega,
+                            const int *S, int L, int lo, int hi, Smem<NT> &, Counters &c) {
+    const int knext = LV::key(L + 1);
+    lv.template prepare_frontier<NT>(S, lo, hi, p.fb_words);
+    auto arc = [&](int x, int y) {
+        if (lv.probe(y) == knext) atomicAdd(&omega[x], omega[y]);  // omega[x] == 0 until finished
+    };
+    ep_scan<NT>(p.src, p.col, p.nnz, lv, L, arc);
+    if (threadIdx.x == 0) c.scanned += (unsigned long long)p.nnz;
     __syncthreads();
     for (int i = lo + threadIdx.x; i < hi; i += NT) {
-        int w = sl.S[i];
-        finish_dependency(p, sl, w, omega[w]);
+        const int w = S[i];
+        finish_dependency(p, sigma, omega, w, omega[w]);
     }
 }
 
 // ------------------------------------------------------------------ kernel
 
-template <bool DIR>
+template <class LV> __device__ __forceinline__ LV make_levels(const KParams &p, size_t slot, uint32_t *dyn);
+template <> __device__ __forceinline__ GlobalLevels make_levels<GlobalLevels>(const KParams &p, size_t slot,
+                                                                              uint32_t *) {
+    GlobalLevels lv;
+    lv.d = p.d + slot * p.stride_n;
+    lv.fb = nullptr;
+    return lv;
+}
+template <> __device__ __forceinline__ SmemCodes make_levels<SmemCodes>(const KParams &p, size_t,
+                                                                        uint32_t *dyn) {
+    SmemCodes lv;
+    lv.w = dyn;
+    lv.fb = dyn + p.code_words;
+    return lv;
+}
+
+template <bool DIR, class LV, int NT>
 __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
-    __shared__ Smem sm;
+    __shared__ Smem<NT> sm;
+    extern __shared__ uint32_t dyn_smem[];
     const size_t slot = blockIdx.x;
-    Slot sl;
-    sl.d = p.d + slot * p.stride_n;
-    sl.sigma = p.sigma + slot * p.stride_n;
-    sl.omega = p.omega + slot * p.stride_n;
-    sl.S = p.S + slot * p.stride_n;
-    sl.ends = p.ends + slot * p.stride_e;
-    sl.modes = p.modes + slot * p.stride_e;
+    const LV lv = make_levels<LV>(p, slot, dyn_smem);
+    double *sigma = p.sigma + slot * p.stride_n;
+    double *omega = p.omega + slot * p.stride_n;
+    int *S = p.S + slot * p.stride_n;
+    int *ends = p.ends + slot * p.stride_e;
+    unsigned char *modes = p.modes + slot * p.stride_e;
 
     Counters c;
     unsigned long long n_src = 0, n_lv = 0, n_we = 0, n_ep = 0, n_reached = 0;
     const int run_ep = (p.launch_mode == LM_SAMPLED && p.sampled_flag) ? *p.sampled_flag : 0;
+    lv.template reset_all<NT>(p.code_words);
 
     for (;;) {
         if (threadIdx.x == 0) sm.idx = (long long)atomicAdd(p.work_counter, 1ULL);
@@ -396,28 +486,28 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
         const long long idx = sm.idx;
         if (idx >= p.k) break;
         const int s = p.sources ? p.sources[p.src_base + idx] : (int)(p.src_base + idx);
-        // Alg. 1; all other entries are already d=INF, sigma=omega=0.
+        // Alg. 1; all other entries are already unvisited / zero.
         if (threadIdx.x == 0) {
-            sl.d[s] = 0;
-            sl.sigma[s] = 1.0;
-            sl.S[0] = s;
-            sl.ends[0] = 0;
-            sl.ends[1] = 1;
+            lv.set_source(s);
+            sigma[s] = 1.0;
+            S[0] = s;
+            ends[0] = 0;
+            ends[1] = 1;
             sm.s_len = 1;
         }
         __syncthreads();
 
         int L = 0, lo = 0, hi = 1;
-        int mode = next_mode(p, MODE_WE, run_ep, 0, 1);  // level 0: frontier = {s}
-        if (p.launch_mode == LM_HYBRID) mode = MODE_WE;  // Alg. 4 starts WE
+        int mode = p.launch_mode == LM_HYBRID ? MODE_WE  // Alg. 4 starts WE
+                                              : next_mode(p, MODE_WE, run_ep, 0, 1);
         for (;;) {
-            if (mode == MODE_WE) forward_we<DIR>(p, sl, L, lo, hi, sm, c);
-            else forward_ep<DIR>(p, sl, L, lo, hi, sm, c);
+            if (mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
+            else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             __syncthreads();
             const int nhi = sm.s_len;
             if (threadIdx.x == 0) {
-                sl.modes[L] = (unsigned char)mode;
-                sl.ends[L + 2] = nhi;
+                modes[L] = (unsigned char)mode;
+                ends[L + 2] = nhi;
             }
             if (mode == MODE_WE) n_we++; else n_ep++;
             n_lv++;
@@ -435,33 +525,39 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
         // Stage 2 (Alg. 3).  Deepest level: delta = 0, omega = 1/sigma.
         if (maxdepth >= 1)
             for (int i = lo + threadIdx.x; i < hi; i += NT) {
-                int v = sl.S[i];
-                sl.omega[v] = 1.0 / sl.sigma[v];
+                const int v = S[i];
+                omega[v] = 1.0 / sigma[v];
             }
         __syncthreads();
         for (int Lb = maxdepth - 1; Lb >= 1; --Lb) {
-            const int blo = sl.ends[Lb], bhi = sl.ends[Lb + 1];
-            const int bmode = p.backward_we ? MODE_WE : (int)sl.modes[Lb];
-            if (bmode == MODE_WE) backward_we(p, sl, Lb, blo, bhi, sm, c);
-            else backward_ep(p, sl, Lb, blo, bhi, sm, c);
+            const int blo = ends[Lb], bhi = ends[Lb + 1];
+            const int bmode = p.backward_we ? MODE_WE : (int)modes[Lb];
+            if (bmode == MODE_WE) backward_we<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
+            else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
             __syncthreads();
         }
 
-        // Debug export, then reset only the touched vertices.
-        for (int i = threadIdx.x; i < S_len; i += NT) {
-            int v = sl.S[i];
-            if (p.dbg_d) {
-                p.dbg_d[v] = sl.d[v];
-                p.dbg_sigma[v] = sl.sigma[v];
+        // Debug export, then reset of the touched state.
+        if (p.dbg_d) {
+            for (int l = 0; l <= maxdepth; ++l)
+                for (int i = ends[l] + threadIdx.x; i < ends[l + 1]; i += NT) {
+                    const int v = S[i];
+                    p.dbg_d[v] = l;
+                    p.dbg_sigma[v] = sigma[v];
+                }
+            if (threadIdx.x == 0) {
+                for (int l = 0; l <= maxdepth && l < p.dbg_max_levels; ++l) p.dbg_modes[l] = modes[l];
+                *p.dbg_nlevels = maxdepth + 1;
             }
-            sl.d[v] = INF;
-            sl.sigma[v] = 0.0;
-            sl.omega[v] = 0.0;
+            __syncthreads();
         }
-        if (p.dbg_modes && threadIdx.x == 0) {
-            for (int l = 0; l <= maxdepth && l < p.dbg_max_levels; ++l) p.dbg_modes[l] = sl.modes[l];
-            *p.dbg_nlevels = maxdepth + 1;
+        for (int i = threadIdx.x; i < S_len; i += NT) {
+            const int v = S[i];
+            lv.reset_vertex(v);
+            sigma[v] = 0.0;
+            omega[v] = 0.0;
         }
+        lv.template reset_all<NT>(p.code_words);
         n_src++;
         n_reached += (unsigned long long)S_len;
         __syncthreads();
@@ -475,7 +571,7 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
         dg += __shfl_down_sync(FULL, dg, o);
         sc += __shfl_down_sync(FULL, sc, o);
     }
-    int inex = __any_sync(FULL, c.inexact);
+    const int inex = __any_sync(FULL, c.inexact);
     if ((threadIdx.x & 31) == 0) {
         atomicAdd(&p.stats->dag_arcs, dg);
         atomicAdd(&p.stats->arcs_scanned, sc);
@@ -504,10 +600,10 @@ __global__ void __launch_bounds__(1024) sampling_decide_kernel(const int *keys, 
     for (int size = 2; size <= P; size <<= 1) {
         for (int stride = size >> 1; stride > 0; stride >>= 1) {
             for (int i = threadIdx.x; i < P; i += blockDim.x) {
-                int j = i ^ stride;
+                const int j = i ^ stride;
                 if (j > i) {
-                    bool up = (i & size) == 0;
-                    int a = sk[i], b = sk[j];
+                    const bool up = (i & size) == 0;
+                    const int a = sk[i], b = sk[j];
                     if ((a > b) == up) { sk[i] = b; sk[j] = a; }
                 }
             }
@@ -515,8 +611,8 @@ __global__ void __launch_bounds__(1024) sampling_decide_kernel(const int *keys, 
         }
     }
     if (threadIdx.x == 0) {
-        int med = sk[nk / 2];
-        int ep = (double)med < thresh ? 1 : 0;
+        const int med = sk[nk / 2];
+        const int ep = (double)med < thresh ? 1 : 0;
         *flag = ep;
         st->sampling_ep = ep;
         st->sampling_median = med;
@@ -528,7 +624,7 @@ __global__ void build_src_kernel(const int *__restrict__ ro, int n, int nnz, int
          a += (long long)gridDim.x * blockDim.x) {
         int lo = 0, hi = n - 1;  // last v with ro[v] <= a
         while (lo < hi) {
-            int mid = (lo + hi + 1) >> 1;
+            const int mid = (lo + hi + 1) >> 1;
             if (ro[mid] <= a) lo = mid; else hi = mid - 1;
         }
         src[a] = lo;

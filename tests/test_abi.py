@@ -55,7 +55,7 @@ def test_struct_layouts_match_header():
 #include "bc.h"
 int main(void){
   printf("%zu %zu %zu %zu\n", sizeof(bc_options), offsetof(bc_options, gamma),
-         offsetof(bc_options, backward_we), sizeof(bc_stats));
+         offsetof(bc_options, level_store), sizeof(bc_stats));
   printf("%zu %zu %zu\n", offsetof(bc_stats, sampling_ep), offsetof(bc_stats, inflight),
          offsetof(bc_stats, kernel_ms));
   return 0; }
@@ -68,7 +68,7 @@ int main(void){
         subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), "-o", exe, c])
         vals = [int(x) for x in subprocess.check_output([exe]).split()]
     O, S = _bc.bc_options, _bc.bc_stats
-    assert vals == [ctypes.sizeof(O), O.gamma.offset, O.backward_we.offset, ctypes.sizeof(S),
+    assert vals == [ctypes.sizeof(O), O.gamma.offset, O.level_store.offset, ctypes.sizeof(S),
                     S.sampling_ep.offset, S.inflight.offset, S.kernel_ms.offset]
 
 
