@@ -30,7 +30,8 @@ class bc_options(ctypes.Structure):
                 ("gamma", ctypes.c_double), ("n_samps", ctypes.c_int32),
                 ("ep_min_frontier", ctypes.c_int32), ("inflight", ctypes.c_int32),
                 ("backward_we", ctypes.c_int32), ("block_threads", ctypes.c_int32),
-                ("seq_max_deg", ctypes.c_int32), ("level_store", ctypes.c_int32)]
+                ("seq_max_deg", ctypes.c_int32), ("level_store", ctypes.c_int32),
+                ("warp_max_deg", ctypes.c_int32), ("l2_persist", ctypes.c_int32)]
 
 
 class bc_stats(ctypes.Structure):
@@ -41,10 +42,12 @@ class bc_stats(ctypes.Structure):
                 ("sampling_ep", ctypes.c_int32), ("sampling_median", ctypes.c_int32),
                 ("sigma_inexact", ctypes.c_int32), ("inflight", ctypes.c_int32),
                 ("kernel_launches", ctypes.c_int32), ("bc_kernel_launches", ctypes.c_int32),
-                ("kernel_ms", ctypes.c_double)]
+                ("kernel_ms", ctypes.c_double), ("phase_cycles", ctypes.c_int64 * 4)]
 
     def as_dict(self):
-        return {k: getattr(self, k) for k, _ in self._fields_}
+        d = {k: getattr(self, k) for k, _ in self._fields_}
+        d["phase_cycles"] = list(self.phase_cycles)
+        return d
 
 
 class BCError(RuntimeError):

@@ -68,7 +68,11 @@ struct bc_graph {
     int use_smem = 0;     // 2-bit level codes in shared memory
     int code_words = 0, fb_words = 0;
     int seq_max_deg = 32;
+    int warp_max_deg = 1024;
     // graph
+    char *graph_buf = nullptr;          // ro | col | src
+    size_t csr_bytes = 0, graph_bytes = 0;
+    cudaAccessPolicyWindow l2win{};     // persisting-L2 window over the CSR (num_bytes 0 = off)
     int *ro = nullptr, *col = nullptr, *src = nullptr;
     int *iro = nullptr, *icol = nullptr, *isrc = nullptr;
     // workspace
@@ -109,6 +113,8 @@ extern "C" void bc_default_options(bc_options *o) {
     o->backward_we = 0;
     o->block_threads = 0;
     o->seq_max_deg = 0;
+    o->warp_max_deg = 0;
+    o->l2_persist = 0;
     o->level_store = 0;
 }
 
@@ -135,7 +141,9 @@ static size_t slot_bytes(const bc_graph *g) {
 
 template <bool DIR, class LV>
 static const void *kernel_for(int nt) {
-    return nt == 512 ? (const void *)bc_kernel<DIR, LV, 512> : (const void *)bc_kernel<DIR, LV, 256>;
+    return nt == 512   ? (const void *)bc_kernel<DIR, LV, 512>
+           : nt == 128 ? (const void *)bc_kernel<DIR, LV, 128>
+                       : (const void *)bc_kernel<DIR, LV, 256>;
 }
 
 // Choose level store, block size and shared memory for both launch kinds
@@ -151,14 +159,35 @@ static int configure(bc_graph *g) {
     g->use_smem = o.level_store == 1 ? 0 : (fits ? 1 : 0);
     int nt = o.block_threads;
     if (nt == 0) nt = 256;
-    if (nt != 256 && nt != 512) return fail(BC_EINVAL, "block_threads must be 0, 256 or 512");
+    if (nt != 128 && nt != 256 && nt != 512)
+        return fail(BC_EINVAL, "block_threads must be 0, 128, 256 or 512");
     g->seq_max_deg = o.seq_max_deg > 0 ? o.seq_max_deg : 32;
+    g->warp_max_deg = std::max(g->seq_max_deg, o.warp_max_deg > 0 ? o.warp_max_deg : 1024);
     g->code_words = g->use_smem ? (int)(code_bytes / 4) : 0;
     g->fb_words = g->use_smem ? (int)(fb_bytes / 4) : 0;
     const void *fn;
     if (g->directed) fn = kernel_for<true, GlobalLevels>(nt);
     else if (g->use_smem) fn = kernel_for<false, SmemCodes>(nt);
     else fn = kernel_for<false, GlobalLevels>(nt);
+    // Persisting-L2 window over the CSR (plus src[] when EP levels can run): every
+    // in-flight source re-reads the same rows, while sigma/omega gathers stream.
+    g->l2win = cudaAccessPolicyWindow{};
+    if (o.l2_persist >= 0 && g->graph_buf) {
+        int max_persist = 0, max_win = 0;
+        CK(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, g->device));
+        CK(cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, g->device));
+        if (max_persist > 0 && max_win > 0) {
+            const size_t span = o.strategy == BC_STRATEGY_WE ? g->csr_bytes : g->graph_bytes;
+            const size_t want = std::min<size_t>(span, (size_t)max_win);
+            const size_t carve = std::min<size_t>(want, (size_t)max_persist);
+            CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve));
+            g->l2win.base_ptr = g->graph_buf;
+            g->l2win.num_bytes = want;
+            g->l2win.hitRatio = (float)((double)carve / (double)want);
+            g->l2win.hitProp = cudaAccessPropertyPersisting;
+            g->l2win.missProp = cudaAccessPropertyStreaming;
+        }
+    }
     g->cfg_we.fn = g->cfg_ep.fn = fn;
     g->cfg_we.nt = g->cfg_ep.nt = nt;
     g->cfg_we.dyn = g->use_smem ? code_bytes : 0;
@@ -205,9 +234,11 @@ extern "C" void bc_destroy(bc_graph *g) {
     DeviceGuard dg(g->device);
     if (g->done) cudaEventSynchronize(g->done);
     free_workspace(g);
-    cudaFree(g->ro);
-    cudaFree(g->col);
-    cudaFree(g->src);
+    if (g->l2win.num_bytes) {
+        cudaCtxResetPersistingL2Cache();
+        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
+    }
+    cudaFree(g->graph_buf);
     cudaFree(g->iro);
     cudaFree(g->icol);
     cudaFree(g->isrc);
@@ -232,9 +263,16 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col) {
     CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&g->done, cudaEventDisableTiming));
     for (auto &e : g->tev) CK(cudaEventCreate(&e));
-    CK(cudaMalloc(&g->ro, sizeof(int) * ((size_t)n + 1)));
-    CK(cudaMalloc(&g->col, sizeof(int) * (size_t)std::max(nnz, 1)));
-    CK(cudaMalloc(&g->src, sizeof(int) * (size_t)std::max(nnz, 1)));
+    // ro | col | src in one allocation so one L2 access-policy window covers the CSR
+    auto al = [](size_t b) { return (b + 255) & ~(size_t)255; };
+    const size_t b_ro = al(sizeof(int) * ((size_t)n + 1));
+    const size_t b_col = al(sizeof(int) * (size_t)std::max(nnz, 1) + 16);
+    CK(cudaMalloc(&g->graph_buf, b_ro + 2 * b_col));
+    g->ro = reinterpret_cast<int *>(g->graph_buf);
+    g->col = reinterpret_cast<int *>(g->graph_buf + b_ro);
+    g->src = reinterpret_cast<int *>(g->graph_buf + b_ro + b_col);
+    g->csr_bytes = b_ro + b_col;
+    g->graph_bytes = b_ro + 2 * b_col;
     CK(cudaMemcpy(g->ro, ro32.data(), sizeof(int) * ((size_t)n + 1), cudaMemcpyHostToDevice));
     if (nnz) CK(cudaMemcpy(g->col, col, sizeof(int) * (size_t)nnz, cudaMemcpyHostToDevice));
     if (nnz && n) {
@@ -319,10 +357,11 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     if (o->strategy < 0 || o->strategy > 3) return fail(BC_EINVAL, "bad strategy %d", o->strategy);
     if (o->n_samps < 1 || o->n_samps > 8192) return fail(BC_EINVAL, "n_samps must be in [1, 8192]");
     if (o->alpha < 0 || o->beta < 0 || o->ep_min_frontier < 0 || o->inflight < 0 || !(o->gamma >= 0) ||
-        o->seq_max_deg < 0 || o->level_store < 0 || o->level_store > 2)
+        o->seq_max_deg < 0 || o->warp_max_deg < 0 || o->level_store < 0 || o->level_store > 2)
         return fail(BC_EINVAL, "invalid parameter");
-    if (o->block_threads != 0 && o->block_threads != 256 && o->block_threads != 512)
-        return fail(BC_EINVAL, "block_threads must be 0, 256 or 512");
+    if (o->block_threads != 0 && o->block_threads != 128 && o->block_threads != 256 &&
+        o->block_threads != 512)
+        return fail(BC_EINVAL, "block_threads must be 0, 128, 256 or 512");
     DeviceGuard dg(g->device);
     if (g->done) CK(cudaEventSynchronize(g->done));
     const bc_options old = g->opt;
@@ -376,6 +415,7 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     p.backward_we = g->opt.backward_we;
     p.code_words = g->code_words;
     p.seq_max_deg = g->seq_max_deg;
+    p.warp_max_deg = g->warp_max_deg;
     p.stats = g->stats;
     p.sampled_flag = g->flag;
     return p;
@@ -390,7 +430,19 @@ static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
     const long long cap = std::min<long long>(g->slots, (long long)c.per_sm * g->num_sms);
     const int grid = (int)std::min<long long>(cap, p.k);
     void *args[] = {&p};
-    CK(cudaLaunchKernel(c.fn, dim3(grid), dim3(c.nt), args, c.dyn, st));
+    cudaLaunchConfig_t lc{};
+    lc.gridDim = dim3(grid);
+    lc.blockDim = dim3(c.nt);
+    lc.dynamicSmemBytes = c.dyn;
+    lc.stream = st;
+    cudaLaunchAttribute attr[1];
+    if (g->l2win.num_bytes) {
+        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[0].val.accessPolicyWindow = g->l2win;
+        lc.attrs = attr;
+        lc.numAttrs = 1;
+    }
+    CK(cudaLaunchKernelExC(&lc, c.fn, args));
     g->last_inflight = std::max(g->last_inflight, grid);
     g->launches++;
     g->bc_launches++;
@@ -612,6 +664,7 @@ extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {
     st->inflight = g->last_inflight;
     st->kernel_launches = g->launches;
     st->bc_kernel_launches = g->bc_launches;
+    for (int q = 0; q < 4; ++q) st->phase_cycles[q] = (int64_t)h.phase_cycles[q];
     st->kernel_ms = 0.0;
     for (int i = 0; i < 2; ++i)
         if (g->tev_used[i]) {

@@ -19,9 +19,9 @@
 //    are summed by one thread in CSR order = the oracle's order (bit-exact).
 //  * the queue is S itself: level L+1 is appended at S[ends[L+1]...] with a
 //    warp-aggregated atomic, so Alg. 2's Q_next -> Q_curr copy disappears.
-//  * rows of degree > seq_max_deg are expanded CTA-cooperatively: block scan of
-//    their degrees, arcs dealt round-robin to all threads, owner found by binary
-//    search in shared memory, warp-segmented reduction of the partial sums.
+//  * rows of degree > seq_max_deg are expanded cooperatively (Merrill et al.'s
+//    scan+warp+CTA gather): one warp per row up to warp_max_deg, the whole
+//    CTA for longer rows, two arcs in flight per thread, one reduction per row.
 //  * EP levels stream src[]/col[] with 16-byte vector loads and test frontier
 //    membership in a shared-memory bitmap.
 //  * backward uses omega[v] = (1 + delta[v]) / sigma[v]: one 8-byte gather per
@@ -43,6 +43,7 @@ enum : int { LM_WE = 0, LM_EP = 1, LM_HYBRID = 2, LM_SAMPLED = 3 };
 struct DevStats {
     unsigned long long sources, levels, we_levels, ep_levels;
     unsigned long long n_reached, arcs_reached, dag_arcs, arcs_scanned;
+    unsigned long long phase_cycles[4];  // SM cycles (CTA thread 0): fwd WE, fwd EP, bwd WE, bwd EP
     int sigma_inexact;
     int sampling_ep;
     int sampling_median;
@@ -75,7 +76,8 @@ struct KParams {
     // shared-memory level codes (SmemCodes): 32-bit words of codes / of the EP bitmap
     int code_words;
     int fb_words;        // 0: this launch never runs an EP level
-    int seq_max_deg;
+    int seq_max_deg;     // rows up to this degree: owner thread, CSR order
+    int warp_max_deg;    // rows up to this degree: one warp; longer: whole CTA
     // strategy
     int launch_mode;
     const int *sampled_flag;  // LM_SAMPLED: 1 = EP run
@@ -92,19 +94,49 @@ struct KParams {
     int *dbg_nlevels;
 };
 
+// Per-thread counters for the byte model / stats, flushed into shared memory once
+// per source (32-bit: at most a few rows' worth of arcs per thread per source).
+struct Counters {
+    unsigned arcs_reached = 0, dag = 0, scanned = 0;
+    int inexact = 0;
+};
+
+// Per-CTA counters in shared memory (updated by thread 0 or by warp leaders).
+struct CtaStats {
+    unsigned long long src, reached, ar, dg, sc;
+    unsigned long long lv[2];   // levels expanded WE / EP
+    unsigned long long cyc[4];  // fwd WE, fwd EP, bwd WE, bwd EP
+    int inexact;
+};
+
+__device__ __forceinline__ void flush_counters(Counters &c, CtaStats &st) {
+    unsigned long long ar = c.arcs_reached, dg = c.dag, sc = c.scanned;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        ar += __shfl_down_sync(0xFFFFFFFFu, ar, o);
+        dg += __shfl_down_sync(0xFFFFFFFFu, dg, o);
+        sc += __shfl_down_sync(0xFFFFFFFFu, sc, o);
+    }
+    const int inex = __any_sync(0xFFFFFFFFu, c.inexact);
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(&st.ar, ar);
+        atomicAdd(&st.dg, dg);
+        atomicAdd(&st.sc, sc);
+        if (inex) st.inexact = 1;
+    }
+    c = Counters{};
+}
+
 template <int NT>
 struct Smem {
     long long idx;
     int s_len;
-    int warp_tot[NT / 32 + 1];
-    int off[NT];
-    int beg[NT];
-    double acc[NT];
-};
-
-struct Counters {
-    unsigned long long arcs_reached = 0, dag = 0, scanned = 0;
-    int inexact = 0;
+    int nbig;             // rows queued for CTA-cooperative expansion in this tile
+    CtaStats st;
+    double red[NT / 32];  // block reduction scratch
+    int big_v[NT];
+    int big_beg[NT];
+    int big_deg[NT];
 };
 
 // ------------------------------------------------------------ level policies
@@ -114,12 +146,12 @@ struct GlobalLevels {
     static constexpr int UNVISITED = INF;
     int *d;
     uint32_t *fb;  // unused
-    __device__ __forceinline__ int probe(int u) const { return d[u]; }
+    __device__ __forceinline__ int probe(int u) const { return __ldcg(&d[u]); }
     __device__ __forceinline__ static int key(int L) { return L; }  // L = -1: matches nothing
     __device__ __forceinline__ bool discover(int u, int L1) const {
         return atomicCAS(&d[u], INF, L1) == INF;
     }
-    __device__ __forceinline__ bool in_frontier(int x, int L) const { return d[x] == L; }
+    __device__ __forceinline__ bool in_frontier(int x, int L) const { return __ldcg(&d[x]) == L; }
     __device__ __forceinline__ void set_source(int s) const { d[s] = 0; }
     __device__ __forceinline__ void reset_vertex(int v) const { d[v] = INF; }
     template <int NT> __device__ __forceinline__ void reset_all(int) const {}
@@ -159,34 +191,6 @@ struct SmemCodes {
 
 // ------------------------------------------------------------------ helpers
 
-template <int NT>
-__device__ __forceinline__ int block_exclusive_scan(int x, int &total, Smem<NT> &sm) {
-    constexpr int NW = NT / 32;
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    int incl = x;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        int y = __shfl_up_sync(FULL, incl, o);
-        if (lane >= o) incl += y;
-    }
-    if (lane == 31) sm.warp_tot[wid] = incl;
-    __syncthreads();
-    if (wid == 0) {
-        int v = lane < NW ? sm.warp_tot[lane] : 0;
-        int inc = v;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            int y = __shfl_up_sync(FULL, inc, o);
-            if (lane >= o) inc += y;
-        }
-        if (lane < NW) sm.warp_tot[lane] = inc - v;
-        if (lane == NW - 1) sm.warp_tot[NW] = inc;
-    }
-    __syncthreads();
-    total = sm.warp_tot[NW];
-    return incl - x + sm.warp_tot[wid];
-}
-
 // Append u to S (Q_next) with one shared atomic per group of converged lanes.
 __device__ __forceinline__ void enqueue(int *S, int *s_len, int u) {
     const unsigned m = __activemask();
@@ -198,30 +202,51 @@ __device__ __forceinline__ void enqueue(int *S, int *s_len, int u) {
     S[base + __popc(m & ((1u << lane) - 1u))] = u;
 }
 
-// Segmented (by non-decreasing owner) warp sum; true for the tail lane of each
-// segment, which then holds the segment total in `val`.
-__device__ __forceinline__ bool warp_segmented_sum(int owner, double &val) {
-    const int lane = threadIdx.x & 31;
+__device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        double v2 = __shfl_up_sync(FULL, val, o);
-        int o2 = __shfl_up_sync(FULL, owner, o);
-        if (lane >= o && o2 == owner) val += v2;
-    }
-    int nxt = __shfl_down_sync(FULL, owner, 1);
-    return owner >= 0 && (lane == 31 || nxt != owner);
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+    return v;
 }
 
-// Row pass over the vertices S[lo, hi): every row [rows[v], rows[v+1]) of `cols`
-// is inspected; op(u, probe(u)) returns a double contribution; finish(v, sum, big)
+// Arcs [b, e) of one row inspected by `lanes` cooperating threads (lane index t),
+// two arcs per thread per step so two gathers are in flight.  Returns this
+// thread's partial sum (fixed decomposition -> deterministic).
+template <class Probe, class Gather, class Visit>
+__device__ __forceinline__ double coop_row(const int *__restrict__ cols, int b, int e, int t,
+                                           int lanes, Probe &probe, Gather &gather, Visit &visit) {
+    double acc = 0.0;
+    for (int a = b + t; a < e; a += 2 * lanes) {
+        const int a2 = a + lanes;
+        const bool has2 = a2 < e;
+        const int u0 = cols[a];
+        const int u1 = has2 ? cols[a2] : u0;
+        const int k0 = probe(u0);
+        const int k1 = probe(u1);
+        const double g0 = gather(u0, k0);
+        const double g1 = has2 ? gather(u1, k1) : 0.0;
+        visit(u0, k0);
+        if (has2) visit(u1, k1);
+        acc += g0;
+        acc += g1;
+    }
+    return acc;
+}
+
+// Row pass over the vertices S[lo, hi) (Merrill et al.'s scan+warp+CTA gather,
+// cited at P:196, with the per-vertex sum the pull needs): every row
+// [rows[v], rows[v+1]) of `cols` is inspected; gather(u, probe(u)) is summed per
+// row, visit(u, probe(u)) performs side effects (discovery), finish(v, sum, coop)
 // is called once per vertex.  Rows of degree <= seq_max are summed by their owner
-// thread in CSR order; longer rows by the whole CTA (load-balanced).
-template <int NT, class Probe, class Op, class Finish>
+// thread in CSR order (the oracle's order); rows up to warp_max by one warp; longer
+// rows by the whole CTA.
+template <int NT, class Probe, class Gather, class Visit, class Finish>
 __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int hi,
                                          const int *__restrict__ rows,
-                                         const int *__restrict__ cols, int seq_max,
-                                         Smem<NT> &sm, Counters &c, Probe probe, Op op,
-                                         Finish finish) {
+                                         const int *__restrict__ cols, int seq_max, int warp_max,
+                                         Smem<NT> &sm, Counters &c, Probe probe, Gather gather,
+                                         Visit visit, Finish finish) {
+    constexpr int NW = NT / 32;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     for (int base = lo; base < hi; base += NT) {
         const int i = base + threadIdx.x;
         int v = -1, beg = 0, deg = 0;
@@ -231,54 +256,75 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             deg = rows[v + 1] - beg;
         }
         c.scanned += deg;
-        const bool big = deg > seq_max;
-        double acc = 0.0;
-        if (v >= 0 && !big) {
+        // (1) short rows: owner thread, CSR order; gathers issued before side effects
+        if (v >= 0 && deg <= seq_max) {
+            double acc = 0.0;
             int a = beg;
             const int e = beg + deg;
             for (; a + 4 <= e; a += 4) {
                 const int u0 = cols[a], u1 = cols[a + 1], u2 = cols[a + 2], u3 = cols[a + 3];
                 const int k0 = probe(u0), k1 = probe(u1), k2 = probe(u2), k3 = probe(u3);
-                acc += op(u0, k0);
-                acc += op(u1, k1);
-                acc += op(u2, k2);
-                acc += op(u3, k3);
+                const double g0 = gather(u0, k0), g1 = gather(u1, k1);
+                const double g2 = gather(u2, k2), g3 = gather(u3, k3);
+                visit(u0, k0);
+                visit(u1, k1);
+                visit(u2, k2);
+                visit(u3, k3);
+                acc += g0;
+                acc += g1;
+                acc += g2;
+                acc += g3;
             }
             for (; a < e; ++a) {
                 const int u = cols[a];
-                acc += op(u, probe(u));
+                const int k = probe(u);
+                acc += gather(u, k);
+                visit(u, k);
             }
+            finish(v, acc, false);
         }
-        int total;
-        const int off = block_exclusive_scan<NT>(big ? deg : 0, total, sm);
-        if (total > 0) {  // block-uniform
-            sm.off[threadIdx.x] = off;
-            sm.beg[threadIdx.x] = beg;
-            sm.acc[threadIdx.x] = 0.0;
+        // (2) medium rows: the lanes of this warp take their rows one at a time
+        unsigned med = __ballot_sync(FULL, v >= 0 && deg > seq_max && deg <= warp_max);
+        while (med) {
+            const int leader = __ffs(med) - 1;
+            med &= med - 1;
+            const int w = __shfl_sync(FULL, v, leader);
+            const int b = __shfl_sync(FULL, beg, leader);
+            const int e = b + __shfl_sync(FULL, deg, leader);
+            const double acc = warp_sum(coop_row(cols, b, e, lane, 32, probe, gather, visit));
+            if (lane == leader) finish(w, acc, true);
+        }
+        // (3) long rows: queued in shared memory, expanded by the whole CTA
+        const bool big = v >= 0 && deg > warp_max;
+        if (__syncthreads_or(big)) {
+            if (big) {
+                const int q = atomicAdd(&sm.nbig, 1);
+                sm.big_v[q] = v;
+                sm.big_beg[q] = beg;
+                sm.big_deg[q] = deg;
+            }
             __syncthreads();
-            for (int jb = 0; jb < total; jb += NT) {
-                const int j = jb + threadIdx.x;
-                int owner = -1;
-                double val = 0.0;
-                if (j < total) {
-                    int lo2 = 0, hi2 = NT - 1;  // last t with off[t] <= j
-#pragma unroll 1
-                    while (lo2 < hi2) {
-                        const int mid = (lo2 + hi2 + 1) >> 1;
-                        if (sm.off[mid] <= j) lo2 = mid; else hi2 = mid - 1;
-                    }
-                    owner = lo2;
-                    const int u = cols[sm.beg[owner] + (j - sm.off[owner])];
-                    val = op(u, probe(u));
+            const int nb = sm.nbig;
+            for (int r = 0; r < nb; ++r) {
+                const int b = sm.big_beg[r];
+                double acc = warp_sum(coop_row(cols, b, b + sm.big_deg[r], threadIdx.x, NT, probe,
+                                               gather, visit));
+                if (lane == 0) sm.red[wid] = acc;
+                __syncthreads();
+                if (threadIdx.x == 0) {
+                    double t = 0.0;
+#pragma unroll
+                    for (int q = 0; q < NW; ++q) t += sm.red[q];
+                    finish(sm.big_v[r], t, true);
                 }
-                if (warp_segmented_sum(owner, val)) atomicAdd(&sm.acc[owner], val);
+                __syncthreads();
             }
+            if (threadIdx.x == 0) sm.nbig = 0;
             __syncthreads();
-            if (big) acc = sm.acc[threadIdx.x];
         }
-        if (v >= 0) finish(v, acc, big);
     }
 }
+
 
 __device__ __forceinline__ int next_mode(const KParams &p, int mode, int run_ep, int q_curr,
                                          int q_next) {
@@ -303,41 +349,40 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
     const int L1 = L + 1;
     const int kprev = LV::key(L - 1);
     auto probe = [&](int u) -> int { return lv.probe(u); };
+    auto pull = [&](int u, int k) -> double { return k == kprev ? __ldcg(&sigma[u]) : 0.0; };
+    auto discover = [&](int u, int k) {
+        if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S, &sm.s_len, u);
+    };
+    auto fin = [&](int v, double acc, bool coop) {
+        sigma[v] = acc;
+        if (coop && acc >= TWO53) c.inexact = 1;
+    };
     if (!DIR) {
         // fused: discovery of level L+1 and sigma pull for level L in one row scan
-        auto op = [&](int u, int k) -> double {
-            if (k == kprev) { c.dag++; return sigma[u]; }
-            if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S, &sm.s_len, u);
-            return 0.0;
+        auto visit = [&](int u, int k) {
+            if (k == kprev) c.dag++;
+            discover(u, k);
         };
-        auto fin = [&](int v, double acc, bool big) {
-            if (L > 0) {
-                sigma[v] = acc;
-                if (big && acc >= TWO53) c.inexact = 1;
-            }
+        auto fin0 = [&](int v, double acc, bool coop) {
+            if (L > 0) fin(v, acc, coop);
         };
-        const unsigned long long before = c.scanned;
-        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, sm, c, probe, op, fin);
+        const unsigned before = c.scanned;
+        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, sm, c, probe, pull,
+                     visit, fin0);
         c.arcs_reached += c.scanned - before;
     } else {
-        auto op1 = [&](int u, int k) -> double {
-            if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S, &sm.s_len, u);
-            return 0.0;
-        };
+        auto none = [&](int, int) -> double { return 0.0; };
         auto fin1 = [&](int, double, bool) {};
-        const unsigned long long before = c.scanned;
-        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, sm, c, probe, op1, fin1);
+        const unsigned before = c.scanned;
+        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, sm, c, probe, none,
+                     discover, fin1);
         c.arcs_reached += c.scanned - before;
         if (L > 0) {
-            auto op2 = [&](int u, int k) -> double {
-                if (k == kprev) { c.dag++; return sigma[u]; }
-                return 0.0;
+            auto count = [&](int, int k) {
+                if (k == kprev) c.dag++;
             };
-            auto fin2 = [&](int v, double acc, bool big) {
-                sigma[v] = acc;
-                if (big && acc >= TWO53) c.inexact = 1;
-            };
-            row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, sm, c, probe, op2, fin2);
+            row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, p.warp_max_deg, sm, c, probe,
+                         pull, count, fin);
         }
     }
 }
@@ -385,25 +430,25 @@ __device__ void forward_ep(const KParams &p, const LV &lv, double *sigma, int *S
         if (k == LV::UNVISITED) {
             if (lv.discover(y, L1)) enqueue(S, &sm.s_len, y);
         } else if (!DIR && k == kprev) {
-            const double s = sigma[y];
+            const double s = __ldcg(&sigma[y]);
             const double old = atomicAdd(&sigma[x], s);
             c.dag++;
             if (old + s >= TWO53) c.inexact = 1;
         }
     };
     ep_scan<NT>(p.src, p.col, p.nnz, lv, L, arc);
-    if (threadIdx.x == 0) c.scanned += (unsigned long long)p.nnz;
+    if (threadIdx.x == 0) sm.st.sc += (unsigned long long)p.nnz;
     if (DIR && L > 0) {
         auto arc_in = [&](int x, int y) {
             if (lv.probe(y) == kprev) {
-                const double s = sigma[y];
+                const double s = __ldcg(&sigma[y]);
                 const double old = atomicAdd(&sigma[x], s);
                 c.dag++;
                 if (old + s >= TWO53) c.inexact = 1;
             }
         };
         ep_scan<NT>(p.isrc, p.icol, p.nnz, lv, L, arc_in);
-        if (threadIdx.x == 0) c.scanned += (unsigned long long)p.nnz;
+        if (threadIdx.x == 0) sm.st.sc += (unsigned long long)p.nnz;
     }
 }
 
@@ -411,7 +456,7 @@ __device__ void forward_ep(const KParams &p, const LV &lv, double *sigma, int *S
 
 __device__ __forceinline__ void finish_dependency(const KParams &p, const double *sigma,
                                                   double *omega, int w, double acc) {
-    const double sw = sigma[w];
+    const double sw = __ldcg(&sigma[w]);
     const double delta = sw * acc;                 // delta[w] = sum sw/sigma[v] (1+delta[v])
     omega[w] = (1.0 + delta) / sw;
     if (delta != 0.0) atomicAdd(&p.bc[w], delta);  // Eq. 3
@@ -423,25 +468,27 @@ __device__ void backward_we(const KParams &p, const LV &lv, const double *sigma,
                             const int *S, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int knext = LV::key(L + 1);
     auto probe = [&](int v) -> int { return lv.probe(v); };
-    auto op = [&](int v, int k) -> double { return k == knext ? omega[v] : 0.0; };
+    auto gather = [&](int v, int k) -> double { return k == knext ? __ldcg(&omega[v]) : 0.0; };
+    auto none = [&](int, int) {};
     auto fin = [&](int w, double acc, bool) { finish_dependency(p, sigma, omega, w, acc); };
-    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, sm, c, probe, op, fin);
+    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, sm, c, probe, gather, none,
+                 fin);
 }
 
 template <int NT, class LV>
 __device__ void backward_ep(const KParams &p, const LV &lv, const double *sigma, double *omega,
-                            const int *S, int L, int lo, int hi, Smem<NT> &, Counters &c) {
+                            const int *S, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int knext = LV::key(L + 1);
     lv.template prepare_frontier<NT>(S, lo, hi, p.fb_words);
     auto arc = [&](int x, int y) {
-        if (lv.probe(y) == knext) atomicAdd(&omega[x], omega[y]);  // omega[x] == 0 until finished
+        if (lv.probe(y) == knext) atomicAdd(&omega[x], __ldcg(&omega[y]));  // omega[x] == 0 until finished
     };
     ep_scan<NT>(p.src, p.col, p.nnz, lv, L, arc);
-    if (threadIdx.x == 0) c.scanned += (unsigned long long)p.nnz;
+    if (threadIdx.x == 0) sm.st.sc += (unsigned long long)p.nnz;
     __syncthreads();
     for (int i = lo + threadIdx.x; i < hi; i += NT) {
         const int w = S[i];
-        finish_dependency(p, sigma, omega, w, omega[w]);
+        finish_dependency(p, sigma, omega, w, __ldcg(&omega[w]));
     }
 }
 
@@ -464,7 +511,7 @@ template <> __device__ __forceinline__ SmemCodes make_levels<SmemCodes>(const KP
 }
 
 template <bool DIR, class LV, int NT>
-__global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
+__global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_kernel(KParams p) {
     __shared__ Smem<NT> sm;
     extern __shared__ uint32_t dyn_smem[];
     const size_t slot = blockIdx.x;
@@ -476,9 +523,12 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
     unsigned char *modes = p.modes + slot * p.stride_e;
 
     Counters c;
-    unsigned long long n_src = 0, n_lv = 0, n_we = 0, n_ep = 0, n_reached = 0;
     const int run_ep = (p.launch_mode == LM_SAMPLED && p.sampled_flag) ? *p.sampled_flag : 0;
     lv.template reset_all<NT>(p.code_words);
+    if (threadIdx.x == 0) {
+        sm.nbig = 0;
+        sm.st = CtaStats{};
+    }
 
     for (;;) {
         if (threadIdx.x == 0) sm.idx = (long long)atomicAdd(p.work_counter, 1ULL);
@@ -501,6 +551,7 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
         int mode = p.launch_mode == LM_HYBRID ? MODE_WE  // Alg. 4 starts WE
                                               : next_mode(p, MODE_WE, run_ep, 0, 1);
         for (;;) {
+            const long long t0 = clock64();
             if (mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             __syncthreads();
@@ -508,9 +559,9 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
             if (threadIdx.x == 0) {
                 modes[L] = (unsigned char)mode;
                 ends[L + 2] = nhi;
+                sm.st.cyc[mode] += (unsigned long long)(clock64() - t0);
+                sm.st.lv[mode] += 1;
             }
-            if (mode == MODE_WE) n_we++; else n_ep++;
-            n_lv++;
             __syncthreads();  // s_len is appended to again by the next level
             if (nhi == hi) break;  // Q_next_len == 0 (Alg. 2 l.11)
             mode = next_mode(p, mode, run_ep, hi - lo, nhi - hi);
@@ -526,15 +577,17 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
         if (maxdepth >= 1)
             for (int i = lo + threadIdx.x; i < hi; i += NT) {
                 const int v = S[i];
-                omega[v] = 1.0 / sigma[v];
+                omega[v] = 1.0 / __ldcg(&sigma[v]);
             }
         __syncthreads();
         for (int Lb = maxdepth - 1; Lb >= 1; --Lb) {
             const int blo = ends[Lb], bhi = ends[Lb + 1];
             const int bmode = p.backward_we ? MODE_WE : (int)modes[Lb];
+            const long long t0 = clock64();
             if (bmode == MODE_WE) backward_we<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
             else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
             __syncthreads();
+            if (threadIdx.x == 0) sm.st.cyc[2 + bmode] += (unsigned long long)(clock64() - t0);
         }
 
         // Debug export, then reset of the touched state.
@@ -543,7 +596,7 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
                 for (int i = ends[l] + threadIdx.x; i < ends[l + 1]; i += NT) {
                     const int v = S[i];
                     p.dbg_d[v] = l;
-                    p.dbg_sigma[v] = sigma[v];
+                    p.dbg_sigma[v] = __ldcg(&sigma[v]);
                 }
             if (threadIdx.x == 0) {
                 for (int l = 0; l <= maxdepth && l < p.dbg_max_levels; ++l) p.dbg_modes[l] = modes[l];
@@ -558,32 +611,27 @@ __global__ void __launch_bounds__(NT) bc_kernel(KParams p) {
             omega[v] = 0.0;
         }
         lv.template reset_all<NT>(p.code_words);
-        n_src++;
-        n_reached += (unsigned long long)S_len;
+        flush_counters(c, sm.st);
+        if (threadIdx.x == 0) {
+            sm.st.src += 1;
+            sm.st.reached += (unsigned long long)S_len;
+        }
         __syncthreads();
     }
 
-    // Statistics: per-thread counters -> warp sums -> global atomics.
-    unsigned long long ar = c.arcs_reached, dg = c.dag, sc = c.scanned;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        ar += __shfl_down_sync(FULL, ar, o);
-        dg += __shfl_down_sync(FULL, dg, o);
-        sc += __shfl_down_sync(FULL, sc, o);
-    }
-    const int inex = __any_sync(FULL, c.inexact);
-    if ((threadIdx.x & 31) == 0) {
-        atomicAdd(&p.stats->dag_arcs, dg);
-        atomicAdd(&p.stats->arcs_scanned, sc);
-        atomicAdd(&p.stats->arcs_reached, ar);
-        if (inex) atomicOr(&p.stats->sigma_inexact, 1);
-    }
     if (threadIdx.x == 0) {
-        atomicAdd(&p.stats->sources, n_src);
-        atomicAdd(&p.stats->levels, n_lv);
-        atomicAdd(&p.stats->we_levels, n_we);
-        atomicAdd(&p.stats->ep_levels, n_ep);
-        atomicAdd(&p.stats->n_reached, n_reached);
+        DevStats *g = p.stats;
+        atomicAdd(&g->sources, sm.st.src);
+        atomicAdd(&g->levels, sm.st.lv[0] + sm.st.lv[1]);
+        atomicAdd(&g->we_levels, sm.st.lv[0]);
+        atomicAdd(&g->ep_levels, sm.st.lv[1]);
+        atomicAdd(&g->n_reached, sm.st.reached);
+        atomicAdd(&g->arcs_reached, sm.st.ar);
+        atomicAdd(&g->dag_arcs, sm.st.dg);
+        atomicAdd(&g->arcs_scanned, sm.st.sc);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) atomicAdd(&g->phase_cycles[q], sm.st.cyc[q]);
+        if (sm.st.inexact) atomicOr(&g->sigma_inexact, 1);
     }
 }
 
