@@ -81,6 +81,8 @@ struct bc_graph {
     double *sigma = nullptr, *omega = nullptr;
     int *S = nullptr, *ends = nullptr;
     unsigned char *modes = nullptr;
+    int *bigq = nullptr;
+    size_t stride_big = 0;
     size_t stride_n = 0, stride_e = 0;
     // per-call buffers
     int *src_buf = nullptr;
@@ -127,6 +129,8 @@ static void free_workspace(bc_graph *g) {
     cudaFree(g->S);
     cudaFree(g->ends);
     cudaFree(g->modes);
+    cudaFree(g->bigq);
+    g->bigq = nullptr;
     g->d = nullptr;
     g->sigma = g->omega = nullptr;
     g->S = g->ends = nullptr;
@@ -136,7 +140,7 @@ static void free_workspace(bc_graph *g) {
 
 static size_t slot_bytes(const bc_graph *g) {
     return g->stride_n * ((g->use_smem ? 0 : sizeof(int)) + 2 * sizeof(double) + sizeof(int)) +
-           g->stride_e * (sizeof(int) + 1);
+           g->stride_e * (sizeof(int) + 1) + g->stride_big * sizeof(int);
 }
 
 template <bool DIR, class LV>
@@ -158,7 +162,13 @@ static int configure(bc_graph *g) {
         return fail(BC_EINVAL, "level_store=2 needs an undirected graph with n <= ~%zu", smem_cap * 8 / 3);
     g->use_smem = o.level_store == 1 ? 0 : (fits ? 1 : 0);
     int nt = o.block_threads;
-    if (nt == 0) nt = 256;
+    if (nt == 0) {
+        // Measured on B200 (tools/sweep.py): dense scale-free graphs want wide CTAs
+        // (frontiers of 10^5 vertices, hub rows), small high-diameter graphs want
+        // many narrow ones (frontiers of a few hundred vertices, more roots in flight).
+        const double avg_deg = g->n ? (double)g->nnz / g->n : 0.0;
+        nt = (g->n >= (1 << 17) && avg_deg >= 16.0) ? 512 : (g->n <= (1 << 16) ? 128 : 256);
+    }
     if (nt != 128 && nt != 256 && nt != 512)
         return fail(BC_EINVAL, "block_threads must be 0, 128, 256 or 512");
     g->seq_max_deg = o.seq_max_deg > 0 ? o.seq_max_deg : 32;
@@ -207,6 +217,8 @@ static int alloc_workspace(bc_graph *g) {
     g->stride_n = (size_t)std::max(g->n, 1);
     g->stride_n = (g->stride_n + 31) & ~(size_t)31;  // 128-byte aligned slots
     g->stride_e = g->stride_n + 32;
+    // a level queues at most nnz / (warp_max + 1) rows for CTA-cooperative expansion
+    g->stride_big = (((size_t)g->nnz / ((size_t)g->warp_max_deg + 1) + 2) + 31) & ~(size_t)31;
     const int occ = std::max(g->cfg_we.per_sm, g->cfg_ep.per_sm) * g->num_sms;
     int want = g->opt.inflight > 0 ? std::min(g->opt.inflight, occ) : occ;
     size_t free_b = 0, total_b = 0;
@@ -222,6 +234,7 @@ static int alloc_workspace(bc_graph *g) {
     CK(cudaMalloc(&g->S, ns * g->stride_n * sizeof(int)));
     CK(cudaMalloc(&g->ends, ns * g->stride_e * sizeof(int)));
     CK(cudaMalloc(&g->modes, ns * g->stride_e));
+    CK(cudaMalloc(&g->bigq, ns * g->stride_big * sizeof(int)));
     if (!g->use_smem) CK(cudaMemset(g->d, 0x7F, ns * g->stride_n * sizeof(int)));  // INF = 0x7F7F7F7F
     CK(cudaMemset(g->sigma, 0, ns * g->stride_n * sizeof(double)));
     CK(cudaMemset(g->omega, 0, ns * g->stride_n * sizeof(double)));
@@ -374,7 +387,7 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     }
     const int old_slots = g->slots;
     const int realloc = o->inflight != old.inflight || o->level_store != old.level_store ||
-                        o->block_threads != old.block_threads;
+                        o->block_threads != old.block_threads || o->warp_max_deg != old.warp_max_deg;
     if (realloc) {
         rc = alloc_workspace(g);
         if (rc) return rc;
@@ -406,6 +419,8 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     p.S = g->S;
     p.ends = g->ends;
     p.modes = g->modes;
+    p.bigq = g->bigq;
+    p.stride_big = g->stride_big;
     p.stride_n = g->stride_n;
     p.stride_e = g->stride_e;
     p.bc = d_bc;

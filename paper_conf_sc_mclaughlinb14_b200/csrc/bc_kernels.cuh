@@ -70,6 +70,8 @@ struct KParams {
     int *S;
     int *ends;
     unsigned char *modes;
+    int *bigq;           // rows queued for CTA-cooperative expansion (per slot)
+    size_t stride_big;
     size_t stride_n;     // elements per slot for d/sigma/omega/S
     size_t stride_e;     // elements per slot for ends/modes
     double *bc;
@@ -209,25 +211,32 @@ __device__ __forceinline__ double warp_sum(double v) {
 }
 
 // Arcs [b, e) of one row inspected by `lanes` cooperating threads (lane index t),
-// two arcs per thread per step so two gathers are in flight.  Returns this
+// four arcs per thread per step so four gathers are in flight.  Returns this
 // thread's partial sum (fixed decomposition -> deterministic).
 template <class Probe, class Gather, class Visit>
 __device__ __forceinline__ double coop_row(const int *__restrict__ cols, int b, int e, int t,
                                            int lanes, Probe &probe, Gather &gather, Visit &visit) {
     double acc = 0.0;
-    for (int a = b + t; a < e; a += 2 * lanes) {
-        const int a2 = a + lanes;
-        const bool has2 = a2 < e;
-        const int u0 = cols[a];
-        const int u1 = has2 ? cols[a2] : u0;
-        const int k0 = probe(u0);
-        const int k1 = probe(u1);
-        const double g0 = gather(u0, k0);
-        const double g1 = has2 ? gather(u1, k1) : 0.0;
+    int a = b + t;
+    for (; a + 3 * lanes < e; a += 4 * lanes) {  // four arcs (and gathers) in flight
+        const int u0 = cols[a], u1 = cols[a + lanes], u2 = cols[a + 2 * lanes], u3 = cols[a + 3 * lanes];
+        const int k0 = probe(u0), k1 = probe(u1), k2 = probe(u2), k3 = probe(u3);
+        const double g0 = gather(u0, k0), g1 = gather(u1, k1);
+        const double g2 = gather(u2, k2), g3 = gather(u3, k3);
         visit(u0, k0);
-        if (has2) visit(u1, k1);
+        visit(u1, k1);
+        visit(u2, k2);
+        visit(u3, k3);
         acc += g0;
         acc += g1;
+        acc += g2;
+        acc += g3;
+    }
+    for (; a < e; a += lanes) {
+        const int u = cols[a];
+        const int k = probe(u);
+        acc += gather(u, k);
+        visit(u, k);
     }
     return acc;
 }
@@ -238,17 +247,19 @@ __device__ __forceinline__ double coop_row(const int *__restrict__ cols, int b, 
 // row, visit(u, probe(u)) performs side effects (discovery), finish(v, sum, coop)
 // is called once per vertex.  Rows of degree <= seq_max are summed by their owner
 // thread in CSR order (the oracle's order); rows up to warp_max by one warp; longer
-// rows by the whole CTA.
+// rows are queued in bigq and expanded by the whole CTA after one barrier.  Warps
+// take 32-vertex chunks independently, so there is no barrier per chunk.
 template <int NT, class Probe, class Gather, class Visit, class Finish>
 __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int hi,
                                          const int *__restrict__ rows,
                                          const int *__restrict__ cols, int seq_max, int warp_max,
-                                         Smem<NT> &sm, Counters &c, Probe probe, Gather gather,
-                                         Visit visit, Finish finish) {
+                                         int *__restrict__ bigq, Smem<NT> &sm, Counters &c,
+                                         Probe probe, Gather gather, Visit visit, Finish finish) {
     constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    for (int base = lo; base < hi; base += NT) {
-        const int i = base + threadIdx.x;
+    // Phase A: each warp walks its own 32-vertex chunks; no CTA barrier.
+    for (int base = lo + wid * 32; base < hi; base += NT) {
+        const int i = base + lane;
         int v = -1, beg = 0, deg = 0;
         if (i < hi) {
             v = S[i];
@@ -294,32 +305,25 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             const double acc = warp_sum(coop_row(cols, b, e, lane, 32, probe, gather, visit));
             if (lane == leader) finish(w, acc, true);
         }
-        // (3) long rows: queued in shared memory, expanded by the whole CTA
-        const bool big = v >= 0 && deg > warp_max;
-        if (__syncthreads_or(big)) {
-            if (big) {
-                const int q = atomicAdd(&sm.nbig, 1);
-                sm.big_v[q] = v;
-                sm.big_beg[q] = beg;
-                sm.big_deg[q] = deg;
-            }
+        // (3) long rows: queued for the CTA-cooperative phase B
+        if (v >= 0 && deg > warp_max) bigq[atomicAdd(&sm.nbig, 1)] = v;
+    }
+    // Phase B: long rows, the whole CTA per row (block reduction of the partials).
+    if (__syncthreads_or(sm.nbig > 0)) {
+        const int nb = sm.nbig;
+        for (int r = 0; r < nb; ++r) {
+            const int v = __ldcg(&bigq[r]);
+            const int b = rows[v], e = rows[v + 1];
+            const double acc = warp_sum(coop_row(cols, b, e, threadIdx.x, NT, probe, gather, visit));
+            if (lane == 0) sm.red[wid] = acc;
             __syncthreads();
-            const int nb = sm.nbig;
-            for (int r = 0; r < nb; ++r) {
-                const int b = sm.big_beg[r];
-                double acc = warp_sum(coop_row(cols, b, b + sm.big_deg[r], threadIdx.x, NT, probe,
-                                               gather, visit));
-                if (lane == 0) sm.red[wid] = acc;
-                __syncthreads();
-                if (threadIdx.x == 0) {
-                    double t = 0.0;
+            if (threadIdx.x == 0) {
+                double t = 0.0;
 #pragma unroll
-                    for (int q = 0; q < NW; ++q) t += sm.red[q];
-                    finish(sm.big_v[r], t, true);
-                }
-                __syncthreads();
+                for (int q = 0; q < NW; ++q) t += sm.red[q];
+                finish(v, t, true);
+                if (r == nb - 1) sm.nbig = 0;  // before the barrier: the next pass may push
             }
-            if (threadIdx.x == 0) sm.nbig = 0;
             __syncthreads();
         }
     }
@@ -344,8 +348,8 @@ __device__ __forceinline__ int next_mode(const KParams &p, int mode, int run_ep,
 // ------------------------------------------------------------------ forward
 
 template <bool DIR, int NT, class LV>
-__device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S, int L, int lo,
-                           int hi, Smem<NT> &sm, Counters &c) {
+__device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S, int *bigq, int L,
+                           int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int L1 = L + 1;
     const int kprev = LV::key(L - 1);
     auto probe = [&](int u) -> int { return lv.probe(u); };
@@ -367,21 +371,21 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
             if (L > 0) fin(v, acc, coop);
         };
         const unsigned before = c.scanned;
-        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, sm, c, probe, pull,
+        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, pull,
                      visit, fin0);
         c.arcs_reached += c.scanned - before;
     } else {
         auto none = [&](int, int) -> double { return 0.0; };
         auto fin1 = [&](int, double, bool) {};
         const unsigned before = c.scanned;
-        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, sm, c, probe, none,
+        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, none,
                      discover, fin1);
         c.arcs_reached += c.scanned - before;
         if (L > 0) {
             auto count = [&](int, int k) {
                 if (k == kprev) c.dag++;
             };
-            row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, p.warp_max_deg, sm, c, probe,
+            row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe,
                          pull, count, fin);
         }
     }
@@ -465,13 +469,14 @@ __device__ __forceinline__ void finish_dependency(const KParams &p, const double
 
 template <int NT, class LV>
 __device__ void backward_we(const KParams &p, const LV &lv, const double *sigma, double *omega,
-                            const int *S, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
+                            const int *S, int *bigq, int L, int lo, int hi, Smem<NT> &sm,
+                            Counters &c) {
     const int knext = LV::key(L + 1);
     auto probe = [&](int v) -> int { return lv.probe(v); };
     auto gather = [&](int v, int k) -> double { return k == knext ? __ldcg(&omega[v]) : 0.0; };
     auto none = [&](int, int) {};
     auto fin = [&](int w, double acc, bool) { finish_dependency(p, sigma, omega, w, acc); };
-    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, sm, c, probe, gather, none,
+    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, gather, none,
                  fin);
 }
 
@@ -521,6 +526,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
     int *S = p.S + slot * p.stride_n;
     int *ends = p.ends + slot * p.stride_e;
     unsigned char *modes = p.modes + slot * p.stride_e;
+    int *bigq = p.bigq + slot * p.stride_big;
 
     Counters c;
     const int run_ep = (p.launch_mode == LM_SAMPLED && p.sampled_flag) ? *p.sampled_flag : 0;
@@ -552,7 +558,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
                                               : next_mode(p, MODE_WE, run_ep, 0, 1);
         for (;;) {
             const long long t0 = clock64();
-            if (mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
+            if (mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             __syncthreads();
             const int nhi = sm.s_len;
@@ -584,7 +590,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
             const int blo = ends[Lb], bhi = ends[Lb + 1];
             const int bmode = p.backward_we ? MODE_WE : (int)modes[Lb];
             const long long t0 = clock64();
-            if (bmode == MODE_WE) backward_we<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
+            if (bmode == MODE_WE) backward_we<NT>(p, lv, sigma, omega, S, bigq, Lb, blo, bhi, sm, c);
             else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
             __syncthreads();
             if (threadIdx.x == 0) sm.st.cyc[2 + bmode] += (unsigned long long)(clock64() - t0);
