@@ -65,7 +65,8 @@ struct bc_graph {
         size_t dyn = 0;   // dynamic shared memory bytes
         int per_sm = 1;   // resident CTAs per SM
     } cfg_we, cfg_ep;
-    int use_smem = 0;     // 2-bit level codes in shared memory
+    int lstore = 1;       // level store: 1 int32 d (HBM), 2 codes in SMEM, 3 codes in HBM/L2
+    uint32_t *gcodes = nullptr, *gfb = nullptr;
     int code_words = 0, fb_words = 0;
     int seq_max_deg = 32;
     int warp_max_deg = 1024;
@@ -75,6 +76,10 @@ struct bc_graph {
     cudaAccessPolicyWindow l2win{};     // persisting-L2 window over the CSR (num_bytes 0 = off)
     int *ro = nullptr, *col = nullptr, *src = nullptr;
     int *iro = nullptr, *icol = nullptr, *isrc = nullptr;
+    // internal relabelling (see want_reorder): perm[old] = new; NULL = identity
+    int *perm = nullptr;
+    std::vector<int> h_perm;
+    double *bc_tmp = nullptr;           // BC in internal ids before mapping back
     // workspace
     int slots = 0;
     int *d = nullptr;
@@ -130,7 +135,10 @@ static void free_workspace(bc_graph *g) {
     cudaFree(g->ends);
     cudaFree(g->modes);
     cudaFree(g->bigq);
+    cudaFree(g->gcodes);
+    cudaFree(g->gfb);
     g->bigq = nullptr;
+    g->gcodes = g->gfb = nullptr;
     g->d = nullptr;
     g->sigma = g->omega = nullptr;
     g->S = g->ends = nullptr;
@@ -139,8 +147,9 @@ static void free_workspace(bc_graph *g) {
 }
 
 static size_t slot_bytes(const bc_graph *g) {
-    return g->stride_n * ((g->use_smem ? 0 : sizeof(int)) + 2 * sizeof(double) + sizeof(int)) +
-           g->stride_e * (sizeof(int) + 1) + g->stride_big * sizeof(int);
+    const size_t gc = g->lstore == 3 ? 4 * ((size_t)g->code_words + (size_t)g->fb_words) : 0;
+    return g->stride_n * ((g->lstore == 1 ? sizeof(int) : 0) + 2 * sizeof(double) + sizeof(int)) +
+           g->stride_e * (sizeof(int) + 1) + g->stride_big * sizeof(int) + gc;
 }
 
 template <bool DIR, class LV>
@@ -154,13 +163,16 @@ static const void *kernel_for(int nt) {
 // (with / without the EP frontier bitmap) and their occupancy.
 static int configure(bc_graph *g) {
     const bc_options &o = g->opt;
-    const size_t code_bytes = (((size_t)g->n + 15) / 16) * 4;
+    const size_t code_bytes = (((size_t)g->n + 63) / 64) * 16;  // words padded to a multiple of 4
     const size_t fb_bytes = (((size_t)g->n + 31) / 32) * 4;
     const size_t smem_cap = 200 * 1024;  // leaves room for the static part (< 16 KB)
     const bool fits = !g->directed && code_bytes + fb_bytes <= smem_cap;
     if (o.level_store == 2 && !fits)
         return fail(BC_EINVAL, "level_store=2 needs an undirected graph with n <= ~%zu", smem_cap * 8 / 3);
-    g->use_smem = o.level_store == 1 ? 0 : (fits ? 1 : 0);
+    if (o.level_store == 3 && g->directed)
+        return fail(BC_EINVAL, "level_store=3 (2-bit codes) needs an undirected graph");
+    if (o.level_store != 0) g->lstore = o.level_store;
+    else g->lstore = g->directed ? 1 : (fits ? 2 : 3);
     int nt = o.block_threads;
     if (nt == 0) {
         // Measured on B200 (tools/sweep.py): dense scale-free graphs want wide CTAs
@@ -173,11 +185,12 @@ static int configure(bc_graph *g) {
         return fail(BC_EINVAL, "block_threads must be 0, 128, 256 or 512");
     g->seq_max_deg = o.seq_max_deg > 0 ? o.seq_max_deg : 32;
     g->warp_max_deg = std::max(g->seq_max_deg, o.warp_max_deg > 0 ? o.warp_max_deg : 1024);
-    g->code_words = g->use_smem ? (int)(code_bytes / 4) : 0;
-    g->fb_words = g->use_smem ? (int)(fb_bytes / 4) : 0;
+    g->code_words = g->lstore >= 2 ? (int)(code_bytes / 4) : 0;
+    g->fb_words = g->lstore >= 2 ? (int)(fb_bytes / 4) : 0;
     const void *fn;
     if (g->directed) fn = kernel_for<true, GlobalLevels>(nt);
-    else if (g->use_smem) fn = kernel_for<false, SmemCodes>(nt);
+    else if (g->lstore == 2) fn = kernel_for<false, SmemCodes>(nt);
+    else if (g->lstore == 3) fn = kernel_for<false, GlobalCodes>(nt);
     else fn = kernel_for<false, GlobalLevels>(nt);
     // Persisting-L2 window over the CSR (plus src[] when EP levels can run): every
     // in-flight source re-reads the same rows, while sigma/omega gathers stream.
@@ -200,8 +213,8 @@ static int configure(bc_graph *g) {
     }
     g->cfg_we.fn = g->cfg_ep.fn = fn;
     g->cfg_we.nt = g->cfg_ep.nt = nt;
-    g->cfg_we.dyn = g->use_smem ? code_bytes : 0;
-    g->cfg_ep.dyn = g->use_smem ? code_bytes + fb_bytes : 0;
+    g->cfg_we.dyn = g->lstore == 2 ? code_bytes : 0;
+    g->cfg_ep.dyn = g->lstore == 2 ? code_bytes + fb_bytes : 0;
     CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_ep.dyn));
     for (auto *c : {&g->cfg_we, &g->cfg_ep}) {
         int per_sm = 0;
@@ -228,14 +241,19 @@ static int alloc_workspace(bc_graph *g) {
     int cap = (int)std::max<size_t>(1, budget / std::max<size_t>(per, 1));
     g->slots = std::max(1, std::min(want, cap));
     size_t ns = (size_t)g->slots;
-    if (!g->use_smem) CK(cudaMalloc(&g->d, ns * g->stride_n * sizeof(int)));
+    if (g->lstore == 1) CK(cudaMalloc(&g->d, ns * g->stride_n * sizeof(int)));
+    if (g->lstore == 3) {
+        CK(cudaMalloc(&g->gcodes, ns * (size_t)g->code_words * 4));
+        CK(cudaMalloc(&g->gfb, ns * (size_t)g->fb_words * 4));
+        CK(cudaMemset(g->gcodes, 0, ns * (size_t)g->code_words * 4));
+    }
     CK(cudaMalloc(&g->sigma, ns * g->stride_n * sizeof(double)));
     CK(cudaMalloc(&g->omega, ns * g->stride_n * sizeof(double)));
     CK(cudaMalloc(&g->S, ns * g->stride_n * sizeof(int)));
     CK(cudaMalloc(&g->ends, ns * g->stride_e * sizeof(int)));
     CK(cudaMalloc(&g->modes, ns * g->stride_e));
     CK(cudaMalloc(&g->bigq, ns * g->stride_big * sizeof(int)));
-    if (!g->use_smem) CK(cudaMemset(g->d, 0x7F, ns * g->stride_n * sizeof(int)));  // INF = 0x7F7F7F7F
+    if (g->lstore == 1) CK(cudaMemset(g->d, 0x7F, ns * g->stride_n * sizeof(int)));  // INF = 0x7F7F7F7F
     CK(cudaMemset(g->sigma, 0, ns * g->stride_n * sizeof(double)));
     CK(cudaMemset(g->omega, 0, ns * g->stride_n * sizeof(double)));
     CK(cudaDeviceSynchronize());
@@ -252,6 +270,8 @@ extern "C" void bc_destroy(bc_graph *g) {
         cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
     }
     cudaFree(g->graph_buf);
+    cudaFree(g->perm);
+    cudaFree(g->bc_tmp);
     cudaFree(g->iro);
     cudaFree(g->icol);
     cudaFree(g->isrc);
@@ -268,11 +288,52 @@ extern "C" void bc_destroy(bc_graph *g) {
     delete g;
 }
 
-static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col) {
+// Internal vertex order.  For skewed degree distributions the vertices are
+// relabelled by descending degree (stable): the sigma/omega entries that the
+// shortest-path DAG gathers most (hub predecessors) then share a few KB per
+// source instead of one 32-byte sector each, and isolated vertices move to the
+// end.  Each row keeps its original neighbour order (so one-thread sums follow
+// the caller's CSR order).  Sources are mapped old -> new on the device and BC is
+// mapped back when it is written out.  BC_REORDER=0/1 overrides the heuristic.
+static bool want_reorder(const bc_graph *g, const int64_t *ro64) {
+    const char *env = getenv("BC_REORDER");
+    if (env && *env) return atoi(env) != 0;
+    if (g->n < 1024) return false;
+    int64_t maxdeg = 0;
+    for (int v = 0; v < g->n; ++v) maxdeg = std::max<int64_t>(maxdeg, ro64[v + 1] - ro64[v]);
+    const double avg = (double)g->nnz / g->n;
+    return (double)maxdeg >= 32.0 * std::max(avg, 1.0);
+}
+
+static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col_in) {
     const int n = g->n;
     const int nnz = g->nnz;
     std::vector<int> ro32((size_t)n + 1);
-    for (int v = 0; v <= n; ++v) ro32[v] = (int)ro64[v];
+    std::vector<int> col_re;
+    const int32_t *col = col_in;
+    if (want_reorder(g, ro64)) {
+        std::vector<int> order((size_t)n);
+        for (int v = 0; v < n; ++v) order[v] = v;
+        std::stable_sort(order.begin(), order.end(), [&](int a, int b) {
+            return ro64[a + 1] - ro64[a] > ro64[b + 1] - ro64[b];
+        });
+        g->h_perm.assign((size_t)n, 0);
+        for (int i = 0; i < n; ++i) g->h_perm[order[i]] = i;  // old -> new
+        col_re.resize((size_t)std::max(nnz, 1));
+        ro32[0] = 0;
+        for (int i = 0; i < n; ++i) {
+            const int v = order[i];
+            int k = ro32[i];
+            for (int64_t e = ro64[v]; e < ro64[v + 1]; ++e) col_re[k++] = g->h_perm[col_in[e]];
+            ro32[i + 1] = k;
+        }
+        col = col_re.data();
+        CK(cudaMalloc(&g->perm, sizeof(int) * (size_t)n));
+        CK(cudaMemcpy(g->perm, g->h_perm.data(), sizeof(int) * (size_t)n, cudaMemcpyHostToDevice));
+        CK(cudaMalloc(&g->bc_tmp, sizeof(double) * (size_t)n));
+    } else {
+        for (int v = 0; v <= n; ++v) ro32[v] = (int)ro64[v];
+    }
     CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&g->done, cudaEventDisableTiming));
     for (auto &e : g->tev) CK(cudaEventCreate(&e));
@@ -370,7 +431,7 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     if (o->strategy < 0 || o->strategy > 3) return fail(BC_EINVAL, "bad strategy %d", o->strategy);
     if (o->n_samps < 1 || o->n_samps > 8192) return fail(BC_EINVAL, "n_samps must be in [1, 8192]");
     if (o->alpha < 0 || o->beta < 0 || o->ep_min_frontier < 0 || o->inflight < 0 || !(o->gamma >= 0) ||
-        o->seq_max_deg < 0 || o->warp_max_deg < 0 || o->level_store < 0 || o->level_store > 2)
+        o->seq_max_deg < 0 || o->warp_max_deg < 0 || o->level_store < 0 || o->level_store > 3)
         return fail(BC_EINVAL, "invalid parameter");
     if (o->block_threads != 0 && o->block_threads != 128 && o->block_threads != 256 &&
         o->block_threads != 512)
@@ -429,10 +490,15 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     p.ep_min_frontier = g->opt.ep_min_frontier;
     p.backward_we = g->opt.backward_we;
     p.code_words = g->code_words;
+    p.gcodes = g->gcodes;
+    p.gfb = g->gfb;
+    p.stride_codes = (size_t)g->code_words;
+    p.stride_fb = (size_t)g->fb_words;
     p.seq_max_deg = g->seq_max_deg;
     p.warp_max_deg = g->warp_max_deg;
     p.stats = g->stats;
     p.sampled_flag = g->flag;
+    p.perm = g->perm;
     return p;
 }
 
@@ -475,13 +541,14 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
         CK(cudaEventRecord(g->done, st));
         return BC_OK;
     }
-    CK(cudaMemsetAsync(d_bc, 0, sizeof(double) * (size_t)g->n, st));
+    double *acc_bc = g->perm ? g->bc_tmp : d_bc;  // accumulate in internal ids
+    CK(cudaMemsetAsync(acc_bc, 0, sizeof(double) * (size_t)g->n, st));
     CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
     CK(cudaMemsetAsync(g->stats, 0, sizeof(DevStats), st));
     g->last_inflight = 0;
     g->launches = g->bc_launches = 0;
     g->tev_used[0] = g->tev_used[1] = 0;
-    KParams p = base_params(g, d_bc);
+    KParams p = base_params(g, acc_bc);
     p.sources = d_sources;
     int rc = BC_OK;
     const int strat = g->opt.strategy;
@@ -534,8 +601,14 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
             g->tev_used[1] = 1;
         }
     }
-    if (!g->directed && g->n > 0) {
-        scale_kernel<<<std::min((g->n + 255) / 256, 148 * 8), 256, 0, st>>>(d_bc, g->n, 0.5);
+    const double h = g->directed ? 1.0 : 0.5;
+    const int eb = std::min((g->n + 255) / 256, 148 * 8);
+    if (g->perm) {
+        unpermute_kernel<<<eb, 256, 0, st>>>(acc_bc, g->perm, g->n, h, d_bc);
+        CK(cudaGetLastError());
+        g->launches++;
+    } else if (!g->directed) {
+        scale_kernel<<<eb, 256, 0, st>>>(d_bc, g->n, h);
         CK(cudaGetLastError());
         g->launches++;
     }
@@ -636,9 +709,21 @@ extern "C" int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigm
     int nl = 0;
     if (rc == BC_OK) {
         e = cudaStreamSynchronize(g->stream);
-        if (e == cudaSuccess && d) e = cudaMemcpy(d, dd, n * sizeof(int), cudaMemcpyDeviceToHost);
-        if (e == cudaSuccess && sigma) e = cudaMemcpy(sigma, ds, n * sizeof(double), cudaMemcpyDeviceToHost);
-        if (e == cudaSuccess && delta) e = cudaMemcpy(delta, ddel, n * sizeof(double), cudaMemcpyDeviceToHost);
+        // the debug arrays are in internal ids: gather them back to the caller's ids
+        const std::vector<int> &pm = g->h_perm;
+        auto fetch = [&](void *host, const void *dev, size_t elem) -> cudaError_t {
+            if (!host) return cudaSuccess;
+            if (!g->perm) return cudaMemcpy(host, dev, n * elem, cudaMemcpyDeviceToHost);
+            std::vector<char> tmp(n * elem);
+            cudaError_t r = cudaMemcpy(tmp.data(), dev, n * elem, cudaMemcpyDeviceToHost);
+            if (r != cudaSuccess) return r;
+            char *h = static_cast<char *>(host);
+            for (size_t v = 0; v < n; ++v) memcpy(h + v * elem, tmp.data() + (size_t)pm[v] * elem, elem);
+            return cudaSuccess;
+        };
+        if (e == cudaSuccess) e = fetch(d, dd, sizeof(int));
+        if (e == cudaSuccess) e = fetch(sigma, ds, sizeof(double));
+        if (e == cudaSuccess) e = fetch(delta, ddel, sizeof(double));
         if (e == cudaSuccess) e = cudaMemcpy(&nl, dn, sizeof(int), cudaMemcpyDeviceToHost);
         if (e == cudaSuccess && level_modes && ml > 0)
             e = cudaMemcpy(level_modes, dm, (size_t)std::min(ml, nl), cudaMemcpyDeviceToHost);

@@ -60,6 +60,7 @@ struct KParams {
     const int *__restrict__ icol;
     const int *__restrict__ isrc;
     const int *__restrict__ sources;  // NULL: source = src_base + idx
+    const int *__restrict__ perm;     // caller id -> internal id (NULL: identity)
     long long src_base;
     long long k;                      // sources in this launch
     unsigned long long *work_counter;
@@ -77,6 +78,9 @@ struct KParams {
     double *bc;
     // shared-memory level codes (SmemCodes): 32-bit words of codes / of the EP bitmap
     int code_words;
+    uint32_t *gcodes;    // GlobalCodes: per-slot code words / EP bitmap words in HBM
+    uint32_t *gfb;
+    size_t stride_codes, stride_fb;
     int fb_words;        // 0: this launch never runs an EP level
     int seq_max_deg;     // rows up to this degree: owner thread, CSR order
     int warp_max_deg;    // rows up to this degree: one warp; longer: whole CTA
@@ -132,7 +136,7 @@ __device__ __forceinline__ void flush_counters(Counters &c, CtaStats &st) {
 template <int NT>
 struct Smem {
     long long idx;
-    int s_len;
+    int cnt[3];           // level L appends at S[hi + cnt[L % 3]] (triple-buffered, see kernel)
     int nbig;             // rows queued for CTA-cooperative expansion in this tile
     CtaStats st;
     double red[NT / 32];  // block reduction scratch
@@ -146,6 +150,7 @@ struct Smem {
 // Exact int32 distances in HBM (directed graphs, or graphs too large for SMEM codes).
 struct GlobalLevels {
     static constexpr int UNVISITED = INF;
+    static constexpr bool RESET_VERTICES = true;
     int *d;
     uint32_t *fb;  // unused
     __device__ __forceinline__ int probe(int u) const { return __ldcg(&d[u]); }
@@ -160,9 +165,51 @@ struct GlobalLevels {
     template <int NT> __device__ __forceinline__ void prepare_frontier(const int *, int, int, int) const {}
 };
 
+// 2-bit level codes in HBM/L2, per slot, for undirected graphs too large for
+// shared memory (n/4 bytes per source: 1 MB at n = 2^22, L2-resident for ~100
+// sources in flight instead of 16 MB of int32 distances).  Same code semantics
+// as SmemCodes; probes bypass L1 (ld.global.cg) because discoveries are atomics.
+struct GlobalCodes {
+    static constexpr int UNVISITED = 0;
+    static constexpr bool RESET_VERTICES = false;
+    uint32_t *w;
+    uint32_t *fb;
+    __device__ __forceinline__ int probe(int u) const {
+        return (__ldcg(&w[u >> 4]) >> ((u & 15) << 1)) & 3;
+    }
+    __device__ __forceinline__ static int key(int L) { return L < 0 ? 4 : (L % 3) + 1; }
+    __device__ __forceinline__ bool discover(int u, int L1) const {
+        const uint32_t sh = (uint32_t)(u & 15) << 1;
+        const uint32_t old = atomicOr(&w[u >> 4], (uint32_t)key(L1) << sh);
+        return ((old >> sh) & 3u) == 0u;
+    }
+    __device__ __forceinline__ bool in_frontier(int x, int) const {
+        return (__ldcg(&fb[x >> 5]) >> (x & 31)) & 1u;
+    }
+    __device__ __forceinline__ void set_source(int s) const {
+        atomicOr(&w[s >> 4], (uint32_t)key(0) << ((s & 15) << 1));
+    }
+    __device__ __forceinline__ void reset_vertex(int) const {}
+    template <int NT> __device__ __forceinline__ void reset_all(int words) const {
+        uint4 *w4 = reinterpret_cast<uint4 *>(w);
+        for (int i = threadIdx.x; i < (words >> 2); i += NT) w4[i] = make_uint4(0u, 0u, 0u, 0u);
+    }
+    template <int NT>
+    __device__ __forceinline__ void prepare_frontier(const int *S, int lo, int hi, int words) const {
+        for (int i = threadIdx.x; i < words; i += NT) fb[i] = 0u;
+        __syncthreads();
+        for (int i = lo + threadIdx.x; i < hi; i += NT) {
+            const int v = S[i];
+            atomicOr(&fb[v >> 5], 1u << (v & 31));
+        }
+        __syncthreads();
+    }
+};
+
 // 2-bit level codes in shared memory, undirected graphs only (see header).
 struct SmemCodes {
     static constexpr int UNVISITED = 0;
+    static constexpr bool RESET_VERTICES = false;
     uint32_t *w;   // codes, 16 vertices per word
     uint32_t *fb;  // EP frontier bitmap, 32 vertices per word
     __device__ __forceinline__ int probe(int u) const { return (w[u >> 4] >> ((u & 15) << 1)) & 3; }
@@ -176,7 +223,8 @@ struct SmemCodes {
     __device__ __forceinline__ void set_source(int s) const { w[s >> 4] |= (uint32_t)key(0) << ((s & 15) << 1); }
     __device__ __forceinline__ void reset_vertex(int) const {}
     template <int NT> __device__ __forceinline__ void reset_all(int words) const {
-        for (int i = threadIdx.x; i < words; i += NT) w[i] = 0u;
+        uint4 *w4 = reinterpret_cast<uint4 *>(w);  // words is a multiple of 4 (host pads)
+        for (int i = threadIdx.x; i < (words >> 2); i += NT) w4[i] = make_uint4(0u, 0u, 0u, 0u);
     }
     // Bitmap of S[lo, hi) (one EP level).  Ends with a barrier.
     template <int NT>
@@ -355,7 +403,7 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
     auto probe = [&](int u) -> int { return lv.probe(u); };
     auto pull = [&](int u, int k) -> double { return k == kprev ? __ldcg(&sigma[u]) : 0.0; };
     auto discover = [&](int u, int k) {
-        if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S, &sm.s_len, u);
+        if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S + hi, &sm.cnt[L % 3], u);
     };
     auto fin = [&](int v, double acc, bool coop) {
         sigma[v] = acc;
@@ -424,15 +472,17 @@ __device__ void forward_ep(const KParams &p, const LV &lv, double *sigma, int *S
                            int hi, Smem<NT> &sm, Counters &c) {
     const int L1 = L + 1;
     const int kprev = LV::key(L - 1);
-    lv.template prepare_frontier<NT>(S, lo, hi, p.fb_words);
-    for (int i = lo + threadIdx.x; i < hi; i += NT) {  // sum of frontier degrees (byte model)
+    for (int i = lo + threadIdx.x; i < hi; i += NT) {
         const int v = S[i];
-        c.arcs_reached += (unsigned long long)(p.ro[v + 1] - p.ro[v]);
+        c.arcs_reached += (unsigned long long)(p.ro[v + 1] - p.ro[v]);  // byte model
+        if (L > 0) sigma[v] = 0.0;  // accumulated with atomics below
     }
+    __syncthreads();
+    lv.template prepare_frontier<NT>(S, lo, hi, p.fb_words);
     auto arc = [&](int x, int y) {
         const int k = lv.probe(y);
         if (k == LV::UNVISITED) {
-            if (lv.discover(y, L1)) enqueue(S, &sm.s_len, y);
+            if (lv.discover(y, L1)) enqueue(S + hi, &sm.cnt[L % 3], y);
         } else if (!DIR && k == kprev) {
             const double s = __ldcg(&sigma[y]);
             const double old = atomicAdd(&sigma[x], s);
@@ -454,6 +504,7 @@ __device__ void forward_ep(const KParams &p, const LV &lv, double *sigma, int *S
         ep_scan<NT>(p.isrc, p.icol, p.nnz, lv, L, arc_in);
         if (threadIdx.x == 0) sm.st.sc += (unsigned long long)p.nnz;
     }
+    __syncthreads();  // every level function ends with a barrier
 }
 
 // ------------------------------------------------------------------ backward
@@ -484,9 +535,11 @@ template <int NT, class LV>
 __device__ void backward_ep(const KParams &p, const LV &lv, const double *sigma, double *omega,
                             const int *S, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int knext = LV::key(L + 1);
+    for (int i = lo + threadIdx.x; i < hi; i += NT) omega[S[i]] = 0.0;  // atomic accumulators
+    __syncthreads();
     lv.template prepare_frontier<NT>(S, lo, hi, p.fb_words);
     auto arc = [&](int x, int y) {
-        if (lv.probe(y) == knext) atomicAdd(&omega[x], __ldcg(&omega[y]));  // omega[x] == 0 until finished
+        if (lv.probe(y) == knext) atomicAdd(&omega[x], __ldcg(&omega[y]));
     };
     ep_scan<NT>(p.src, p.col, p.nnz, lv, L, arc);
     if (threadIdx.x == 0) sm.st.sc += (unsigned long long)p.nnz;
@@ -495,6 +548,7 @@ __device__ void backward_ep(const KParams &p, const LV &lv, const double *sigma,
         const int w = S[i];
         finish_dependency(p, sigma, omega, w, __ldcg(&omega[w]));
     }
+    __syncthreads();  // every level function ends with a barrier
 }
 
 // ------------------------------------------------------------------ kernel
@@ -514,11 +568,18 @@ template <> __device__ __forceinline__ SmemCodes make_levels<SmemCodes>(const KP
     lv.fb = dyn + p.code_words;
     return lv;
 }
+template <> __device__ __forceinline__ GlobalCodes make_levels<GlobalCodes>(const KParams &p, size_t slot,
+                                                                            uint32_t *) {
+    GlobalCodes lv;
+    lv.w = p.gcodes + slot * p.stride_codes;
+    lv.fb = p.gfb + slot * p.stride_fb;
+    return lv;
+}
 
 template <bool DIR, class LV, int NT>
 __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_kernel(KParams p) {
     __shared__ Smem<NT> sm;
-    extern __shared__ uint32_t dyn_smem[];
+    extern __shared__ __align__(16) uint32_t dyn_smem[];
     const size_t slot = blockIdx.x;
     const LV lv = make_levels<LV>(p, slot, dyn_smem);
     double *sigma = p.sigma + slot * p.stride_n;
@@ -541,7 +602,8 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
         __syncthreads();
         const long long idx = sm.idx;
         if (idx >= p.k) break;
-        const int s = p.sources ? p.sources[p.src_base + idx] : (int)(p.src_base + idx);
+        int s = p.sources ? p.sources[p.src_base + idx] : (int)(p.src_base + idx);
+        if (p.perm) s = p.perm[s];  // caller's id -> internal id
         // Alg. 1; all other entries are already unvisited / zero.
         if (threadIdx.x == 0) {
             lv.set_source(s);
@@ -549,7 +611,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
             S[0] = s;
             ends[0] = 0;
             ends[1] = 1;
-            sm.s_len = 1;
+            sm.cnt[0] = sm.cnt[1] = sm.cnt[2] = 0;
         }
         __syncthreads();
 
@@ -560,15 +622,17 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
             const long long t0 = clock64();
             if (mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
-            __syncthreads();
-            const int nhi = sm.s_len;
+            // (the level functions end with a barrier: every discovery is appended)
+            const int nhi = hi + sm.cnt[L % 3];
             if (threadIdx.x == 0) {
                 modes[L] = (unsigned char)mode;
                 ends[L + 2] = nhi;
+                // cnt[(L+2)%3] was last used by level L-1 and read by every thread
+                // before level L started; it is next used by level L+2.
+                sm.cnt[(L + 2) % 3] = 0;
                 sm.st.cyc[mode] += (unsigned long long)(clock64() - t0);
                 sm.st.lv[mode] += 1;
             }
-            __syncthreads();  // s_len is appended to again by the next level
             if (nhi == hi) break;  // Q_next_len == 0 (Alg. 2 l.11)
             mode = next_mode(p, mode, run_ep, hi - lo, nhi - hi);
             lo = hi;
@@ -592,7 +656,6 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
             const long long t0 = clock64();
             if (bmode == MODE_WE) backward_we<NT>(p, lv, sigma, omega, S, bigq, Lb, blo, bhi, sm, c);
             else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
-            __syncthreads();
             if (threadIdx.x == 0) sm.st.cyc[2 + bmode] += (unsigned long long)(clock64() - t0);
         }
 
@@ -610,12 +673,10 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
             }
             __syncthreads();
         }
-        for (int i = threadIdx.x; i < S_len; i += NT) {
-            const int v = S[i];
-            lv.reset_vertex(v);
-            sigma[v] = 0.0;
-            omega[v] = 0.0;
-        }
+        // sigma / omega need no reset: every entry is written before it is read
+        // (pull writes sigma[w], finish writes omega[w]; EP zeroes its accumulators).
+        if (LV::RESET_VERTICES)
+            for (int i = threadIdx.x; i < S_len; i += NT) lv.reset_vertex(S[i]);
         lv.template reset_all<NT>(p.code_words);
         flush_counters(c, sm.st);
         if (threadIdx.x == 0) {
@@ -689,6 +750,14 @@ __global__ void scale_kernel(double *bc, int n, double f) {
     for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
          i += (long long)gridDim.x * blockDim.x)
         bc[i] *= f;
+}
+
+// out[v] = f * bc_internal[perm[v]]: back to the caller's vertex ids (and halving).
+__global__ void unpermute_kernel(const double *__restrict__ bc_int, const int *__restrict__ perm,
+                                 int n, double f, double *__restrict__ out) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+         i += (long long)gridDim.x * blockDim.x)
+        out[i] = f * bc_int[perm[i]];
 }
 
 }  // namespace bcdev

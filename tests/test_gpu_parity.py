@@ -324,3 +324,32 @@ def test_multi_shard_sum_equals_whole(bcmod, oracle_mod):
         for P in (2, 3, 8):
             parts = [bg.compute(dist.shard_sources(S, r, P, seed=4)) for r in range(P)]
             assert rel_err(np.sum(parts, axis=0), whole) <= 1e-12
+
+
+@pytest.mark.parametrize("reorder", ["0", "1"])
+def test_internal_reordering_is_invisible(bcmod, oracle_mod, monkeypatch, reorder):
+    """The degree-ordered internal relabelling (BC_REORDER) must not change any
+    output: BC, d, sigma, delta and the per-level modes are in the caller's ids."""
+    monkeypatch.setenv("BC_REORDER", reorder)
+    for g in (graph("c1"), gg.gnp(300, 0.02, seed=3, directed=True), gg.star_graph(500)):
+        with bcmod.BCGraph.from_graph(g, strategy="sampling", ep_min_frontier=1) as bg:
+            src = gg.sample_sources(g, min(200, int((g.degrees() > 0).sum())), seed=1)
+            check_bc(bg, g, src, oracle_mod)
+            check_bc(bg, g, None, oracle_mod)
+            for s in src[:5]:
+                check_source(bg, g, s, oracle_mod)
+
+
+@pytest.mark.parametrize("level_store", [1, 2, 3])
+@pytest.mark.parametrize("strategy", ["we", "sampling"])
+def test_level_stores_agree(bcmod, oracle_mod, level_store, strategy):
+    """Exact int32 d in HBM (1), 2-bit codes in shared memory (2) and 2-bit codes
+    in HBM/L2 (3) are interchangeable representations of d."""
+    for key, k in (("c1", None), ("c4", 300)):
+        g = graph(key)
+        src = None if k is None else gg.CONFIGS[key].sources(g)[:k]
+        with bcmod.BCGraph.from_graph(g, strategy=strategy, level_store=level_store,
+                                      ep_min_frontier=64) as bg:
+            check_bc(bg, g, src, oracle_mod)
+            s0 = int(src[0]) if src is not None else 7
+            check_source(bg, g, s0, oracle_mod)
