@@ -69,7 +69,7 @@ struct bc_graph {
     uint32_t *gcodes = nullptr, *gfb = nullptr;
     int code_words = 0, fb_words = 0;
     int seq_max_deg = 32;
-    int warp_max_deg = 1024;
+    int warp_max_deg = 4096;
     // graph
     char *graph_buf = nullptr;          // ro | col | src
     size_t csr_bytes = 0, graph_bytes = 0;
@@ -152,11 +152,20 @@ static size_t slot_bytes(const bc_graph *g) {
            g->stride_e * (sizeof(int) + 1) + g->stride_big * sizeof(int) + gc;
 }
 
-template <bool DIR, class LV>
+template <bool DIR, class LV, bool EPOK>
 static const void *kernel_for(int nt) {
-    return nt == 512   ? (const void *)bc_kernel<DIR, LV, 512>
-           : nt == 128 ? (const void *)bc_kernel<DIR, LV, 128>
-                       : (const void *)bc_kernel<DIR, LV, 256>;
+    return nt == 1024  ? (const void *)bc_kernel<DIR, LV, 1024, EPOK>
+           : nt == 512 ? (const void *)bc_kernel<DIR, LV, 512, EPOK>
+           : nt == 128 ? (const void *)bc_kernel<DIR, LV, 128, EPOK>
+                       : (const void *)bc_kernel<DIR, LV, 256, EPOK>;
+}
+
+template <bool EPOK>
+static const void *pick_kernel(const bc_graph *g, int nt) {
+    if (g->directed) return kernel_for<true, GlobalLevels, EPOK>(nt);
+    if (g->lstore == 2) return kernel_for<false, SmemCodes, EPOK>(nt);
+    if (g->lstore == 3) return kernel_for<false, GlobalCodes, EPOK>(nt);
+    return kernel_for<false, GlobalLevels, EPOK>(nt);
 }
 
 // Choose level store, block size and shared memory for both launch kinds
@@ -175,23 +184,18 @@ static int configure(bc_graph *g) {
     else g->lstore = g->directed ? 1 : (fits ? 2 : 3);
     int nt = o.block_threads;
     if (nt == 0) {
-        // Measured on B200 (tools/sweep.py): dense scale-free graphs want wide CTAs
-        // (frontiers of 10^5 vertices, hub rows), small high-diameter graphs want
-        // many narrow ones (frontiers of a few hundred vertices, more roots in flight).
-        const double avg_deg = g->n ? (double)g->nnz / g->n : 0.0;
-        nt = (g->n >= (1 << 17) && avg_deg >= 16.0) ? 512 : (g->n <= (1 << 16) ? 128 : 256);
+        // Measured on B200 (tools/sweep.py): graphs of 2^17+ vertices (frontiers of
+        // 10^3..10^5 vertices, hub rows) want wide CTAs; small graphs want many
+        // narrow ones (frontiers of a few hundred vertices, more roots in flight).
+        nt = g->n >= (1 << 17) ? 512 : 128;
     }
-    if (nt != 128 && nt != 256 && nt != 512)
-        return fail(BC_EINVAL, "block_threads must be 0, 128, 256 or 512");
+    if (nt != 128 && nt != 256 && nt != 512 && nt != 1024)
+        return fail(BC_EINVAL, "block_threads must be 0, 128, 256, 512 or 1024");
     g->seq_max_deg = o.seq_max_deg > 0 ? o.seq_max_deg : 32;
-    g->warp_max_deg = std::max(g->seq_max_deg, o.warp_max_deg > 0 ? o.warp_max_deg : 1024);
+    g->warp_max_deg = std::max(g->seq_max_deg, o.warp_max_deg > 0 ? o.warp_max_deg : 4096);
     g->code_words = g->lstore >= 2 ? (int)(code_bytes / 4) : 0;
     g->fb_words = g->lstore >= 2 ? (int)(fb_bytes / 4) : 0;
-    const void *fn;
-    if (g->directed) fn = kernel_for<true, GlobalLevels>(nt);
-    else if (g->lstore == 2) fn = kernel_for<false, SmemCodes>(nt);
-    else if (g->lstore == 3) fn = kernel_for<false, GlobalCodes>(nt);
-    else fn = kernel_for<false, GlobalLevels>(nt);
+
     // Persisting-L2 window over the CSR (plus src[] when EP levels can run): every
     // in-flight source re-reads the same rows, while sigma/omega gathers stream.
     g->l2win = cudaAccessPolicyWindow{};
@@ -211,11 +215,13 @@ static int configure(bc_graph *g) {
             g->l2win.missProp = cudaAccessPropertyStreaming;
         }
     }
-    g->cfg_we.fn = g->cfg_ep.fn = fn;
+    g->cfg_we.fn = pick_kernel<false>(g, nt);
+    g->cfg_ep.fn = pick_kernel<true>(g, nt);
     g->cfg_we.nt = g->cfg_ep.nt = nt;
     g->cfg_we.dyn = g->lstore == 2 ? code_bytes : 0;
     g->cfg_ep.dyn = g->lstore == 2 ? code_bytes + fb_bytes : 0;
-    CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_ep.dyn));
+    CK(cudaFuncSetAttribute(g->cfg_we.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_we.dyn));
+    CK(cudaFuncSetAttribute(g->cfg_ep.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_ep.dyn));
     for (auto *c : {&g->cfg_we, &g->cfg_ep}) {
         int per_sm = 0;
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, c->fn, c->nt, c->dyn));
@@ -434,8 +440,8 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
         o->seq_max_deg < 0 || o->warp_max_deg < 0 || o->level_store < 0 || o->level_store > 3)
         return fail(BC_EINVAL, "invalid parameter");
     if (o->block_threads != 0 && o->block_threads != 128 && o->block_threads != 256 &&
-        o->block_threads != 512)
-        return fail(BC_EINVAL, "block_threads must be 0, 128, 256 or 512");
+        o->block_threads != 512 && o->block_threads != 1024)
+        return fail(BC_EINVAL, "block_threads must be 0, 128, 256, 512 or 1024");
     DeviceGuard dg(g->device);
     if (g->done) CK(cudaEventSynchronize(g->done));
     const bc_options old = g->opt;

@@ -24,8 +24,8 @@
 //    CTA for longer rows, two arcs in flight per thread, one reduction per row.
 //  * EP levels stream src[]/col[] with 16-byte vector loads and test frontier
 //    membership in a shared-memory bitmap.
-//  * backward uses omega[v] = (1 + delta[v]) / sigma[v]: one 8-byte gather per
-//    DAG arc, delta[w] = sigma[w] * sum(omega of successors).
+//  * backward uses omega[v] = (1 + delta[v]) / sigma[v], stored in place of
+//    sigma[v]: one 8-byte gather per DAG arc, delta[w] = sigma[w] * sum(omega).
 #pragma once
 
 #include <cstdint>
@@ -265,26 +265,25 @@ template <class Probe, class Gather, class Visit>
 __device__ __forceinline__ double coop_row(const int *__restrict__ cols, int b, int e, int t,
                                            int lanes, Probe &probe, Gather &gather, Visit &visit) {
     double acc = 0.0;
-    int a = b + t;
-    for (; a + 3 * lanes < e; a += 4 * lanes) {  // four arcs (and gathers) in flight
-        const int u0 = cols[a], u1 = cols[a + lanes], u2 = cols[a + 2 * lanes], u3 = cols[a + 3 * lanes];
+    for (int a = b + t; a < e; a += 4 * lanes) {  // four arcs (and gathers) in flight
+        const bool v1 = a + lanes < e, v2 = a + 2 * lanes < e, v3 = a + 3 * lanes < e;
+        const int u0 = cols[a];
+        const int u1 = v1 ? cols[a + lanes] : u0;
+        const int u2 = v2 ? cols[a + 2 * lanes] : u0;
+        const int u3 = v3 ? cols[a + 3 * lanes] : u0;
         const int k0 = probe(u0), k1 = probe(u1), k2 = probe(u2), k3 = probe(u3);
-        const double g0 = gather(u0, k0), g1 = gather(u1, k1);
-        const double g2 = gather(u2, k2), g3 = gather(u3, k3);
+        const double g0 = gather(u0, k0);
+        const double g1 = v1 ? gather(u1, k1) : 0.0;
+        const double g2 = v2 ? gather(u2, k2) : 0.0;
+        const double g3 = v3 ? gather(u3, k3) : 0.0;
         visit(u0, k0);
-        visit(u1, k1);
-        visit(u2, k2);
-        visit(u3, k3);
+        if (v1) visit(u1, k1);
+        if (v2) visit(u2, k2);
+        if (v3) visit(u3, k3);
         acc += g0;
         acc += g1;
         acc += g2;
         acc += g3;
-    }
-    for (; a < e; a += lanes) {
-        const int u = cols[a];
-        const int k = probe(u);
-        acc += gather(u, k);
-        visit(u, k);
     }
     return acc;
 }
@@ -297,12 +296,13 @@ __device__ __forceinline__ double coop_row(const int *__restrict__ cols, int b, 
 // thread in CSR order (the oracle's order); rows up to warp_max by one warp; longer
 // rows are queued in bigq and expanded by the whole CTA after one barrier.  Warps
 // take 32-vertex chunks independently, so there is no barrier per chunk.
-template <int NT, class Probe, class Gather, class Visit, class Finish>
+template <int NT, class Probe, class Gather, class Visit, class Pre, class Finish>
 __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int hi,
                                          const int *__restrict__ rows,
                                          const int *__restrict__ cols, int seq_max, int warp_max,
                                          int *__restrict__ bigq, Smem<NT> &sm, Counters &c,
-                                         Probe probe, Gather gather, Visit visit, Finish finish) {
+                                         Probe probe, Gather gather, Visit visit, Pre pre,
+                                         Finish finish) {
     constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     // Phase A: each warp walks its own 32-vertex chunks; no CTA barrier.
@@ -317,30 +317,30 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
         c.scanned += deg;
         // (1) short rows: owner thread, CSR order; gathers issued before side effects
         if (v >= 0 && deg <= seq_max) {
+            const double pv = pre(v);
             double acc = 0.0;
-            int a = beg;
             const int e = beg + deg;
-            for (; a + 4 <= e; a += 4) {
-                const int u0 = cols[a], u1 = cols[a + 1], u2 = cols[a + 2], u3 = cols[a + 3];
+            for (int a = beg; a < e; a += 4) {  // CSR order; +0.0 for padding slots
+                const bool v1 = a + 1 < e, v2 = a + 2 < e, v3 = a + 3 < e;
+                const int u0 = cols[a];
+                const int u1 = v1 ? cols[a + 1] : u0;
+                const int u2 = v2 ? cols[a + 2] : u0;
+                const int u3 = v3 ? cols[a + 3] : u0;
                 const int k0 = probe(u0), k1 = probe(u1), k2 = probe(u2), k3 = probe(u3);
-                const double g0 = gather(u0, k0), g1 = gather(u1, k1);
-                const double g2 = gather(u2, k2), g3 = gather(u3, k3);
+                const double g0 = gather(u0, k0);
+                const double g1 = v1 ? gather(u1, k1) : 0.0;
+                const double g2 = v2 ? gather(u2, k2) : 0.0;
+                const double g3 = v3 ? gather(u3, k3) : 0.0;
                 visit(u0, k0);
-                visit(u1, k1);
-                visit(u2, k2);
-                visit(u3, k3);
+                if (v1) visit(u1, k1);
+                if (v2) visit(u2, k2);
+                if (v3) visit(u3, k3);
                 acc += g0;
                 acc += g1;
                 acc += g2;
                 acc += g3;
             }
-            for (; a < e; ++a) {
-                const int u = cols[a];
-                const int k = probe(u);
-                acc += gather(u, k);
-                visit(u, k);
-            }
-            finish(v, acc, false);
+            finish(v, acc, false, pv);
         }
         // (2) medium rows: the lanes of this warp take their rows one at a time
         unsigned med = __ballot_sync(FULL, v >= 0 && deg > seq_max && deg <= warp_max);
@@ -350,8 +350,9 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             const int w = __shfl_sync(FULL, v, leader);
             const int b = __shfl_sync(FULL, beg, leader);
             const int e = b + __shfl_sync(FULL, deg, leader);
+            const double pv = pre(w);
             const double acc = warp_sum(coop_row(cols, b, e, lane, 32, probe, gather, visit));
-            if (lane == leader) finish(w, acc, true);
+            if (lane == leader) finish(w, acc, true, pv);
         }
         // (3) long rows: queued for the CTA-cooperative phase B
         if (v >= 0 && deg > warp_max) bigq[atomicAdd(&sm.nbig, 1)] = v;
@@ -362,6 +363,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
         for (int r = 0; r < nb; ++r) {
             const int v = __ldcg(&bigq[r]);
             const int b = rows[v], e = rows[v + 1];
+            const double pv = pre(v);
             const double acc = warp_sum(coop_row(cols, b, e, threadIdx.x, NT, probe, gather, visit));
             if (lane == 0) sm.red[wid] = acc;
             __syncthreads();
@@ -369,7 +371,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
                 double t = 0.0;
 #pragma unroll
                 for (int q = 0; q < NW; ++q) t += sm.red[q];
-                finish(v, t, true);
+                finish(v, t, true, pv);
                 if (r == nb - 1) sm.nbig = 0;  // before the barrier: the next pass may push
             }
             __syncthreads();
@@ -405,36 +407,37 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
     auto discover = [&](int u, int k) {
         if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S + hi, &sm.cnt[L % 3], u);
     };
-    auto fin = [&](int v, double acc, bool coop) {
+    auto fin = [&](int v, double acc, bool coop, double) {
         sigma[v] = acc;
         if (coop && acc >= TWO53) c.inexact = 1;
     };
+    auto nopre = [&](int) -> double { return 0.0; };
     if (!DIR) {
         // fused: discovery of level L+1 and sigma pull for level L in one row scan
         auto visit = [&](int u, int k) {
             if (k == kprev) c.dag++;
             discover(u, k);
         };
-        auto fin0 = [&](int v, double acc, bool coop) {
-            if (L > 0) fin(v, acc, coop);
+        auto fin0 = [&](int v, double acc, bool coop, double) {
+            if (L > 0) fin(v, acc, coop, 0.0);
         };
         const unsigned before = c.scanned;
         row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, pull,
-                     visit, fin0);
+                     visit, nopre, fin0);
         c.arcs_reached += c.scanned - before;
     } else {
         auto none = [&](int, int) -> double { return 0.0; };
-        auto fin1 = [&](int, double, bool) {};
+        auto fin1 = [&](int, double, bool, double) {};
         const unsigned before = c.scanned;
         row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, none,
-                     discover, fin1);
+                     discover, nopre, fin1);
         c.arcs_reached += c.scanned - before;
         if (L > 0) {
             auto count = [&](int, int k) {
                 if (k == kprev) c.dag++;
             };
             row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe,
-                         pull, count, fin);
+                         pull, count, nopre, fin);
         }
     }
 }
@@ -448,9 +451,7 @@ __device__ __forceinline__ void ep_scan(const int *__restrict__ a_src, const int
     const int n4 = nnz >> 2;
     const int4 *s4 = reinterpret_cast<const int4 *>(a_src);
     const int4 *d4 = reinterpret_cast<const int4 *>(a_dst);
-#pragma unroll 2
-    for (int q = threadIdx.x; q < n4; q += NT) {
-        const int4 xs = s4[q];
+    auto quad = [&](const int4 xs, int q) {
         const bool f0 = lv.in_frontier(xs.x, L), f1 = lv.in_frontier(xs.y, L);
         const bool f2 = lv.in_frontier(xs.z, L), f3 = lv.in_frontier(xs.w, L);
         if (f0 | f1 | f2 | f3) {
@@ -460,6 +461,18 @@ __device__ __forceinline__ void ep_scan(const int *__restrict__ a_src, const int
             if (f2) arc(xs.z, ys.z);
             if (f3) arc(xs.w, ys.w);
         }
+    };
+    const int4 none = make_int4(0, 0, 0, 0);
+    for (int q = threadIdx.x; q < n4; q += 4 * NT) {  // four 16-byte src loads in flight
+        const bool v1 = q + NT < n4, v2 = q + 2 * NT < n4, v3 = q + 3 * NT < n4;
+        const int4 x0 = s4[q];
+        const int4 x1 = v1 ? s4[q + NT] : none;
+        const int4 x2 = v2 ? s4[q + 2 * NT] : none;
+        const int4 x3 = v3 ? s4[q + 3 * NT] : none;
+        quad(x0, q);
+        if (v1) quad(x1, q + NT);
+        if (v2) quad(x2, q + 2 * NT);
+        if (v3) quad(x3, q + 3 * NT);
     }
     for (int a = (n4 << 2) + threadIdx.x; a < nnz; a += NT) {
         const int x = a_src[a];
@@ -484,10 +497,8 @@ __device__ void forward_ep(const KParams &p, const LV &lv, double *sigma, int *S
         if (k == LV::UNVISITED) {
             if (lv.discover(y, L1)) enqueue(S + hi, &sm.cnt[L % 3], y);
         } else if (!DIR && k == kprev) {
-            const double s = __ldcg(&sigma[y]);
-            const double old = atomicAdd(&sigma[x], s);
+            atomicAdd(&sigma[x], __ldcg(&sigma[y]));  // result unused -> RED (no return trip)
             c.dag++;
-            if (old + s >= TWO53) c.inexact = 1;
         }
     };
     ep_scan<NT>(p.src, p.col, p.nnz, lv, L, arc);
@@ -495,58 +506,63 @@ __device__ void forward_ep(const KParams &p, const LV &lv, double *sigma, int *S
     if (DIR && L > 0) {
         auto arc_in = [&](int x, int y) {
             if (lv.probe(y) == kprev) {
-                const double s = __ldcg(&sigma[y]);
-                const double old = atomicAdd(&sigma[x], s);
+                atomicAdd(&sigma[x], __ldcg(&sigma[y]));
                 c.dag++;
-                if (old + s >= TWO53) c.inexact = 1;
             }
         };
         ep_scan<NT>(p.isrc, p.icol, p.nnz, lv, L, arc_in);
         if (threadIdx.x == 0) sm.st.sc += (unsigned long long)p.nnz;
     }
+    __syncthreads();
+    // atomic (order-dependent) sums that reached 2^53 may differ in the last bits
+    for (int i = lo + threadIdx.x; i < hi; i += NT)
+        if (__ldcg(&sigma[S[i]]) >= TWO53) c.inexact = 1;
     __syncthreads();  // every level function ends with a barrier
 }
 
 // ------------------------------------------------------------------ backward
 
-__device__ __forceinline__ void finish_dependency(const KParams &p, const double *sigma,
-                                                  double *omega, int w, double acc) {
-    const double sw = __ldcg(&sigma[w]);
+// omega[w] = (1 + delta[w]) / sigma[w] is stored IN PLACE of sigma[w]: sigma[w]
+// is only needed to finish w itself, and every gather of the backward stage
+// reads a vertex one level deeper, whose entry already holds omega.  One f64
+// array per source instead of two (smaller working set in L2).
+__device__ __forceinline__ void finish_dependency(const KParams &p, double sw, double *sig_om,
+                                                  int w, double acc) {
     const double delta = sw * acc;                 // delta[w] = sum sw/sigma[v] (1+delta[v])
-    omega[w] = (1.0 + delta) / sw;
+    sig_om[w] = (1.0 + delta) / sw;
     if (delta != 0.0) atomicAdd(&p.bc[w], delta);  // Eq. 3
     if (p.dbg_delta) p.dbg_delta[w] = delta;
 }
 
 template <int NT, class LV>
-__device__ void backward_we(const KParams &p, const LV &lv, const double *sigma, double *omega,
-                            const int *S, int *bigq, int L, int lo, int hi, Smem<NT> &sm,
-                            Counters &c) {
+__device__ void backward_we(const KParams &p, const LV &lv, double *sig_om, const int *S, int *bigq,
+                            int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int knext = LV::key(L + 1);
     auto probe = [&](int v) -> int { return lv.probe(v); };
-    auto gather = [&](int v, int k) -> double { return k == knext ? __ldcg(&omega[v]) : 0.0; };
+    auto gather = [&](int v, int k) -> double { return k == knext ? __ldcg(&sig_om[v]) : 0.0; };
     auto none = [&](int, int) {};
-    auto fin = [&](int w, double acc, bool) { finish_dependency(p, sigma, omega, w, acc); };
+    auto pre = [&](int w) -> double { return __ldcg(&sig_om[w]); };  // sigma[w], issued early
+    auto fin = [&](int w, double acc, bool, double sw) { finish_dependency(p, sw, sig_om, w, acc); };
     row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, gather, none,
-                 fin);
+                 pre, fin);
 }
 
 template <int NT, class LV>
-__device__ void backward_ep(const KParams &p, const LV &lv, const double *sigma, double *omega,
+__device__ void backward_ep(const KParams &p, const LV &lv, double *sig_om, double *acc_ep,
                             const int *S, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int knext = LV::key(L + 1);
-    for (int i = lo + threadIdx.x; i < hi; i += NT) omega[S[i]] = 0.0;  // atomic accumulators
+    for (int i = lo + threadIdx.x; i < hi; i += NT) acc_ep[S[i]] = 0.0;  // atomic accumulators
     __syncthreads();
     lv.template prepare_frontier<NT>(S, lo, hi, p.fb_words);
     auto arc = [&](int x, int y) {
-        if (lv.probe(y) == knext) atomicAdd(&omega[x], __ldcg(&omega[y]));
+        if (lv.probe(y) == knext) atomicAdd(&acc_ep[x], __ldcg(&sig_om[y]));
     };
     ep_scan<NT>(p.src, p.col, p.nnz, lv, L, arc);
     if (threadIdx.x == 0) sm.st.sc += (unsigned long long)p.nnz;
     __syncthreads();
     for (int i = lo + threadIdx.x; i < hi; i += NT) {
         const int w = S[i];
-        finish_dependency(p, sigma, omega, w, __ldcg(&omega[w]));
+        finish_dependency(p, __ldcg(&sig_om[w]), sig_om, w, __ldcg(&acc_ep[w]));
     }
     __syncthreads();  // every level function ends with a barrier
 }
@@ -576,8 +592,11 @@ template <> __device__ __forceinline__ GlobalCodes make_levels<GlobalCodes>(cons
     return lv;
 }
 
-template <bool DIR, class LV, int NT>
-__global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_kernel(KParams p) {
+// EPOK = false instantiates a work-efficient-only kernel (no EP code, fewer
+// registers) for launches that never run an EP level.
+template <bool DIR, class LV, int NT, bool EPOK>
+__global__ void __launch_bounds__(NT, NT >= 1024 ? 1 : (NT == 512 ? 2 : (NT == 256 ? 4 : 8)))
+bc_kernel(KParams p) {
     __shared__ Smem<NT> sm;
     extern __shared__ __align__(16) uint32_t dyn_smem[];
     const size_t slot = blockIdx.x;
@@ -620,7 +639,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
                                               : next_mode(p, MODE_WE, run_ep, 0, 1);
         for (;;) {
             const long long t0 = clock64();
-            if (mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, L, lo, hi, sm, c);
+            if (!EPOK || mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             // (the level functions end with a barrier: every discovery is appended)
             const int nhi = hi + sm.cnt[L % 3];
@@ -643,30 +662,32 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
         const int S_len = hi;
         if (p.keys && threadIdx.x == 0) p.keys[idx] = maxdepth;
 
-        // Stage 2 (Alg. 3).  Deepest level: delta = 0, omega = 1/sigma.
-        if (maxdepth >= 1)
-            for (int i = lo + threadIdx.x; i < hi; i += NT) {
-                const int v = S[i];
-                omega[v] = 1.0 / __ldcg(&sigma[v]);
-            }
-        __syncthreads();
-        for (int Lb = maxdepth - 1; Lb >= 1; --Lb) {
-            const int blo = ends[Lb], bhi = ends[Lb + 1];
-            const int bmode = p.backward_we ? MODE_WE : (int)modes[Lb];
-            const long long t0 = clock64();
-            if (bmode == MODE_WE) backward_we<NT>(p, lv, sigma, omega, S, bigq, Lb, blo, bhi, sm, c);
-            else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
-            if (threadIdx.x == 0) sm.st.cyc[2 + bmode] += (unsigned long long)(clock64() - t0);
-        }
-
-        // Debug export, then reset of the touched state.
-        if (p.dbg_d) {
+        if (p.dbg_d) {  // debug export of d and sigma before omega overwrites sigma
             for (int l = 0; l <= maxdepth; ++l)
                 for (int i = ends[l] + threadIdx.x; i < ends[l + 1]; i += NT) {
                     const int v = S[i];
                     p.dbg_d[v] = l;
                     p.dbg_sigma[v] = __ldcg(&sigma[v]);
                 }
+        }
+        // Stage 2 (Alg. 3).  Deepest level: delta = 0, omega = 1/sigma (in place).
+        if (maxdepth >= 1)
+            for (int i = lo + threadIdx.x; i < hi; i += NT) {
+                const int v = S[i];
+                sigma[v] = 1.0 / __ldcg(&sigma[v]);
+            }
+        __syncthreads();
+        for (int Lb = maxdepth - 1; Lb >= 1; --Lb) {
+            const int blo = ends[Lb], bhi = ends[Lb + 1];
+            const int bmode = p.backward_we ? MODE_WE : (int)modes[Lb];
+            const long long t0 = clock64();
+            if (!EPOK || bmode == MODE_WE) backward_we<NT>(p, lv, sigma, S, bigq, Lb, blo, bhi, sm, c);
+            else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
+            if (threadIdx.x == 0) sm.st.cyc[2 + bmode] += (unsigned long long)(clock64() - t0);
+        }
+
+        // Debug export, then reset of the touched state.
+        if (p.dbg_d) {
             if (threadIdx.x == 0) {
                 for (int l = 0; l <= maxdepth && l < p.dbg_max_levels; ++l) p.dbg_modes[l] = modes[l];
                 *p.dbg_nlevels = maxdepth + 1;
@@ -674,7 +695,8 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : (NT == 256 ? 4 : 8)) bc_ke
             __syncthreads();
         }
         // sigma / omega need no reset: every entry is written before it is read
-        // (pull writes sigma[w], finish writes omega[w]; EP zeroes its accumulators).
+        // (pull writes sigma[w], finish overwrites it with omega; EP zeroes its
+        // accumulators).
         if (LV::RESET_VERTICES)
             for (int i = threadIdx.x; i < S_len; i += NT) lv.reset_vertex(S[i]);
         lv.template reset_all<NT>(p.code_words);

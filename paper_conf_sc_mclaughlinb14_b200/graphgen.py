@@ -19,8 +19,11 @@ undirected edges = nnz/2.
 """
 from __future__ import annotations
 
+import ctypes
 import dataclasses
 import math
+import os
+import subprocess
 from typing import Callable, Dict, Optional
 
 import numpy as np
@@ -47,12 +50,69 @@ class Graph:
         return np.diff(self.row_offsets)
 
 
+# ------------------------------------------------------------------ native part
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_NATIVE_SRC = os.path.join(_HERE, "graphgen_native.c")
+_NATIVE_LIB = os.path.join(_HERE, "libgraphgen.so")
+_native = None
+
+
+def _threads() -> int:
+    return max(1, min(32, len(os.sched_getaffinity(0))))
+
+
+def native():
+    """graphgen_native.c (gcc -O2, built on first use): counter-based R-MAT edge
+    draw and a threaded CSR builder.  Input generation only."""
+    global _native
+    if _native is None:
+        if (not os.path.exists(_NATIVE_LIB)
+                or os.path.getmtime(_NATIVE_LIB) < os.path.getmtime(_NATIVE_SRC)):
+            tmp = _NATIVE_LIB + f".{os.getpid()}.tmp"
+            subprocess.check_call(["gcc", "-O2", "-std=c99", "-fPIC", "-shared", "-pthread",
+                                   "-o", tmp, _NATIVE_SRC])
+            os.replace(tmp, _NATIVE_LIB)
+        lib = ctypes.CDLL(_NATIVE_LIB)
+        i64p = ctypes.POINTER(ctypes.c_int64)
+        lib.gg_rmat_edges.argtypes = [ctypes.c_int, ctypes.c_int64, ctypes.c_double, ctypes.c_double,
+                                      ctypes.c_double, ctypes.c_uint64, i64p, i64p, ctypes.c_int]
+        lib.gg_rmat_edges.restype = None
+        lib.gg_permutation.argtypes = [ctypes.c_int64, ctypes.c_uint64, i64p]
+        lib.gg_permutation.restype = None
+        lib.gg_csr_build.argtypes = [ctypes.c_int64, ctypes.c_int64, i64p, i64p, ctypes.c_int, i64p,
+                                     ctypes.POINTER(ctypes.c_int32), ctypes.c_int]
+        lib.gg_csr_build.restype = ctypes.c_int64
+        _native = lib
+    return _native
+
+
+def _p64(a):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_int64))
+
+
 # --------------------------------------------------------------------------- CSR
 
 
 def csr_from_edges(n: int, u: np.ndarray, v: np.ndarray, directed: bool = False,
                    name: str = "graph") -> Graph:
-    """Build a simple-graph CSR: drop self-loops, (symmetrise), dedupe, sort rows."""
+    """Build a simple-graph CSR: drop self-loops, (symmetrise), dedupe, sort rows
+    (threaded C builder; csr_from_edges_numpy is the reference it is tested against)."""
+    u = np.ascontiguousarray(u, dtype=np.int64)
+    v = np.ascontiguousarray(v, dtype=np.int64)
+    cap = u.size if directed else 2 * u.size
+    ro = np.zeros(n + 1, dtype=np.int64)
+    col = np.empty(max(cap, 1), dtype=np.int32)
+    nnz = native().gg_csr_build(int(n), int(u.size), _p64(u), _p64(v), int(directed), _p64(ro),
+                                col.ctypes.data_as(ctypes.POINTER(ctypes.c_int32)), _threads())
+    if nnz < 0:
+        raise ValueError("edge endpoint out of range (or out of memory)")
+    return Graph(name=name, n=n, row_offsets=ro, col_indices=col[:nnz].copy(), directed=directed)
+
+
+def csr_from_edges_numpy(n: int, u: np.ndarray, v: np.ndarray, directed: bool = False,
+                         name: str = "graph") -> Graph:
+    """Reference numpy CSR builder (same contract as csr_from_edges)."""
     u = np.asarray(u, dtype=np.int64)
     v = np.asarray(v, dtype=np.int64)
     if u.size:
@@ -74,6 +134,23 @@ def csr_from_edges(n: int, u: np.ndarray, v: np.ndarray, directed: bool = False,
 # --------------------------------------------------------------------- generators
 
 
+def rmat_edges(scale: int, edgefactor: int = 16, a: float = 0.57, b: float = 0.19,
+               c: float = 0.19, seed: int = 1, relabel: bool = True):
+    """Raw R-MAT edge list (u, v) before the CSR builder; edge i is a pure function
+    of (seed, i) (counter-based splitmix64 draw, graphgen_native.c)."""
+    n = 1 << scale
+    ne = edgefactor * n
+    u = np.empty(ne, dtype=np.int64)
+    v = np.empty(ne, dtype=np.int64)
+    lib = native()
+    lib.gg_rmat_edges(scale, ne, a, b, c, seed & 0xFFFFFFFFFFFFFFFF, _p64(u), _p64(v), _threads())
+    if relabel:
+        perm = np.empty(n, dtype=np.int64)
+        lib.gg_permutation(n, seed & 0xFFFFFFFFFFFFFFFF, _p64(perm))
+        u, v = perm[u], perm[v]
+    return n, u, v
+
+
 def rmat(scale: int, edgefactor: int = 16, a: float = 0.57, b: float = 0.19,
          c: float = 0.19, seed: int = 1, relabel: bool = True,
          directed: bool = False, name: Optional[str] = None) -> Graph:
@@ -84,32 +161,7 @@ def rmat(scale: int, edgefactor: int = 16, a: float = 0.57, b: float = 0.19,
     then randomly permuted.  Duplicates and self-loops are removed by the CSR
     builder (so m < edgefactor*n, and many vertices are isolated).
     """
-    n = 1 << scale
-    ne = edgefactor * n
-    rng = np.random.default_rng(seed)
-    ab = a + b
-    c_norm = c / (1.0 - ab)
-    a_norm = a / ab
-    us, vs = [], []
-    chunk = 1 << 22
-    for lo in range(0, ne, chunk):
-        cnt = min(chunk, ne - lo)
-        u = np.zeros(cnt, dtype=np.int64)
-        v = np.zeros(cnt, dtype=np.int64)
-        for bit in range(scale):
-            r1 = rng.random(cnt)
-            r2 = rng.random(cnt)
-            ii = r1 > ab
-            jj = r2 > np.where(ii, c_norm, a_norm)
-            u |= ii.astype(np.int64) << bit
-            v |= jj.astype(np.int64) << bit
-        us.append(u)
-        vs.append(v)
-    u = np.concatenate(us)
-    v = np.concatenate(vs)
-    if relabel:
-        perm = rng.permutation(n).astype(np.int64)
-        u, v = perm[u], perm[v]
+    n, u, v = rmat_edges(scale, edgefactor, a, b, c, seed, relabel)
     return csr_from_edges(n, u, v, directed=directed,
                           name=name or f"rmat_s{scale}_ef{edgefactor}")
 

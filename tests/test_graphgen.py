@@ -92,3 +92,34 @@ def test_sources():
     assert np.array_equal(gg.sample_sources(g, None, 0), np.arange(g.n))
     p = gg.permute_sources(s, 2)
     assert np.array_equal(np.sort(p), s)
+
+
+@pytest.mark.parametrize("directed", [False, True])
+def test_native_csr_builder_matches_numpy_reference(directed):
+    n, u, v = gg.rmat_edges(11, 16, seed=9)
+    u = np.concatenate([u, [3, 5]])          # explicit self-loop and duplicate
+    v = np.concatenate([v, [3, int(v[0])]])
+    u[-1] = u[0]
+    a = gg.csr_from_edges(n, u, v, directed=directed)
+    b = gg.csr_from_edges_numpy(n, u, v, directed=directed)
+    assert np.array_equal(a.row_offsets, b.row_offsets)
+    assert np.array_equal(a.col_indices, b.col_indices)
+    check_csr(a)
+    with pytest.raises(ValueError):
+        gg.csr_from_edges(4, np.array([0]), np.array([4]))
+
+
+def test_rmat_edges_are_counter_based():
+    """Edge i depends only on (seed, i): a longer draw extends a shorter one."""
+    _, u1, v1 = gg.rmat_edges(8, 4, seed=3, relabel=False)
+    _, u2, v2 = gg.rmat_edges(8, 8, seed=3, relabel=False)
+    assert np.array_equal(u1, u2[:u1.size]) and np.array_equal(v1, v2[:v1.size])
+
+
+def test_kron_s22_calibration_numbers():
+    """m ~ 64.15M, ~42.9 % isolated, max degree ~163k (seeded draw)."""
+    g = gg.CONFIGS["c5k"].graph()
+    d = g.degrees()
+    assert abs(g.m - 64.15e6) / 64.15e6 < 0.01
+    assert 0.40 < (d == 0).mean() < 0.46
+    assert 100_000 < d.max() < 250_000

@@ -18,6 +18,7 @@ def main():
     ap.add_argument("--sources", type=int, default=0, help="0 = the config's source set")
     ap.add_argument("--repeat", type=int, default=1)
     ap.add_argument("--opt", action="append", default=[], help="option=value")
+    ap.add_argument("--stats-out", default=None, help="write the step's stats + byte model as JSON")
     a = ap.parse_args()
     import torch
     import paper_conf_sc_mclaughlinb14_b200 as bcm
@@ -37,6 +38,14 @@ def main():
     st = bg.stats()
     print({k: st[k] for k in ("sources", "levels", "ep_levels", "kernel_ms", "n_reached",
                               "arcs_reached", "dag_arcs", "inflight")}, file=sys.stderr)
+    if a.stats_out:
+        import json
+        # SURVEY 8(d) byte model, per launch-step (all bc_kernel launches of the step)
+        alg = (20.0 * g.n * st["sources"] + 16.0 * st["arcs_reached"] + 24.0 * st["dag_arcs"]
+               + 64.0 * st["n_reached"])
+        json.dump({"config": a.config, "strategy": a.strategy, "sources": int(src.size),
+                   "stats": st, "alg_bytes_per_step": alg, "launches": st["bc_kernel_launches"]},
+                  open(a.stats_out, "w"), indent=1)
     bg.close()
 
 
