@@ -19,6 +19,12 @@ through the host-buffer C-ABI call bc_compute (host sources in, host BC out).
 `roofline` uses the algorithmic byte model of SURVEY §8(d) with the per-source
 counts returned by the kernel, against MEASURED_PEAKS.json's HBM bandwidth.
 `cpu_baseline` (and --impl reference) time the CPU oracle on this host.
+
+Strategy: the paper's sampling selector (Alg. 5) with its EP guard
+("designed to scale with the architecture") retuned for B200 by the
+ablation in profiles/r01/ablation_v1.json: on B200 the
+work-efficient expansion beats edge-parallel at every frontier size measured, so
+the tuned guard admits no EP level.  --paper-params restores guard = 512.
 """
 from __future__ import annotations
 
@@ -192,10 +198,23 @@ def run_reference(args):
     return 0
 
 
+# N1 retune (profiles/r01/ablation_v1.json): EP lost to WE at every frontier size on
+# B200, so the tuned guard exceeds any frontier (no EP level is admitted).
+B200_EP_GUARD = 2147483647
+
+
+def bench_options(args):
+    o = {"strategy": args.strategy}
+    if args.strategy == "sampling":
+        o["ep_min_frontier"] = 512 if args.paper_params else int(args.ep_guard)
+    return o
+
+
 def workload_config(cfg, g, total, world, args):
     return {"workload": f"{cfg.key}: {cfg.description}", "graph": g.name, "n": g.n, "m": g.m,
             "sources_total": int(total.size), "sources_per_gpu": int(math.ceil(total.size / world)),
-            "strategy": args.strategy, "parallelism": f"sources split over {world} GPU(s)",
+            "strategy": args.strategy, "options": bench_options(args),
+            "parallelism": f"sources split over {world} GPU(s)",
             "l2": "flushed before every timed step (256 MiB write)", "seed": cfg.seed}
 
 
@@ -218,7 +237,7 @@ def run_ours(args):
     cfg, g, total, local = make_workload(args.config, world, rank, args.scaling)
     log(f"rank {rank}: graph {g.name} n={g.n} m={g.m} local sources {local.size} "
         f"(gen {time.time() - t0:.1f}s)")
-    bg = bcm.BCGraph.from_graph(g, device=local_rank, strategy=args.strategy)
+    bg = bcm.BCGraph.from_graph(g, device=local_rank, **bench_options(args))
     stream = torch.cuda.Stream(dev)
     d_src = torch.from_numpy(local).to(dev)
     out = torch.zeros(g.n, dtype=torch.float64, device=dev)
@@ -358,6 +377,10 @@ def main():
     ap.add_argument("--config", default="c4")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--strategy", default="sampling", choices=["we", "ep", "hybrid", "sampling"])
+    ap.add_argument("--ep-guard", type=int, default=B200_EP_GUARD,
+                    help="Alg. 5 EP guard (min frontier for an EP level); paper: 512")
+    ap.add_argument("--paper-params", action="store_true",
+                    help="use the paper's EP guard (512) instead of the B200-retuned one")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -69,6 +69,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     global _lib
     if _lib is not None:
         return _lib
+    path = os.environ.get("BC_LIBBC", path)  # alternative build (tuning experiments)
     if not os.path.exists(path):
         raise RuntimeError(f"{path} not found: build it with `make` or __graft_entry__.build()")
     lib = ctypes.CDLL(path)

@@ -511,7 +511,13 @@ static KParams base_params(bc_graph *g, double *d_bc) {
 static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
     if (p0.k <= 0) return BC_OK;
     KParams p = p0;
-    const bool ep_possible = p.launch_mode != LM_WE;
+    // An EP level needs a frontier of >= ep_min_frontier (Alg. 5 guard) or > beta
+    // (Alg. 4) vertices; when no frontier can be that large, the work-efficient-only
+    // kernel (no EP code, no bitmap) is launched instead.
+    const bool ep_possible =
+        p.launch_mode == LM_EP ||
+        (p.launch_mode == LM_SAMPLED && (long long)p.ep_min_frontier <= (long long)g->n) ||
+        (p.launch_mode == LM_HYBRID && (long long)p.beta < (long long)g->n);
     const bc_graph::KCfg &c = ep_possible ? g->cfg_ep : g->cfg_we;
     p.fb_words = ep_possible ? g->fb_words : 0;
     const long long cap = std::min<long long>(g->slots, (long long)c.per_sm * g->num_sms);

@@ -258,32 +258,38 @@ __device__ __forceinline__ double warp_sum(double v) {
     return v;
 }
 
-// Arcs [b, e) of one row inspected by `lanes` cooperating threads (lane index t),
-// four arcs per thread per step so four gathers are in flight.  Returns this
-// thread's partial sum (fixed decomposition -> deterministic).
-template <class Probe, class Gather, class Visit>
-__device__ __forceinline__ double coop_row(const int *__restrict__ cols, int b, int e, int t,
-                                           int lanes, Probe &probe, Gather &gather, Visit &visit) {
+#ifndef BC_UNROLL
+#define BC_UNROLL 4
+#endif
+
+// Arcs a, a+stride, ... < e of one row: stride 1 for a row owned by one thread
+// (CSR order), stride = #cooperating threads for warp/CTA rows.  BC_UNROLL arcs
+// per step so that many col loads and gathers are in flight; padding slots add
+// +0.0, which leaves the CSR-order sum bit-identical.
+template <int U, class Probe, class Gather, class Visit>
+__device__ __forceinline__ double strided_sum(const int *__restrict__ cols, int a, int e, int stride,
+                                              Probe &probe, Gather &gather, Visit &visit) {
     double acc = 0.0;
-    for (int a = b + t; a < e; a += 4 * lanes) {  // four arcs (and gathers) in flight
-        const bool v1 = a + lanes < e, v2 = a + 2 * lanes < e, v3 = a + 3 * lanes < e;
-        const int u0 = cols[a];
-        const int u1 = v1 ? cols[a + lanes] : u0;
-        const int u2 = v2 ? cols[a + 2 * lanes] : u0;
-        const int u3 = v3 ? cols[a + 3 * lanes] : u0;
-        const int k0 = probe(u0), k1 = probe(u1), k2 = probe(u2), k3 = probe(u3);
-        const double g0 = gather(u0, k0);
-        const double g1 = v1 ? gather(u1, k1) : 0.0;
-        const double g2 = v2 ? gather(u2, k2) : 0.0;
-        const double g3 = v3 ? gather(u3, k3) : 0.0;
-        visit(u0, k0);
-        if (v1) visit(u1, k1);
-        if (v2) visit(u2, k2);
-        if (v3) visit(u3, k3);
-        acc += g0;
-        acc += g1;
-        acc += g2;
-        acc += g3;
+    for (; a < e; a += U * stride) {
+        int u[U], k[U];
+        bool ok[U];
+        double g[U];
+        u[0] = cols[a];
+        ok[0] = true;
+#pragma unroll
+        for (int j = 1; j < U; ++j) {
+            ok[j] = a + j * stride < e;
+            u[j] = ok[j] ? cols[a + j * stride] : u[0];
+        }
+#pragma unroll
+        for (int j = 0; j < U; ++j) k[j] = probe(u[j]);
+#pragma unroll
+        for (int j = 0; j < U; ++j) g[j] = ok[j] ? gather(u[j], k[j]) : 0.0;
+#pragma unroll
+        for (int j = 0; j < U; ++j)
+            if (ok[j]) visit(u[j], k[j]);
+#pragma unroll
+        for (int j = 0; j < U; ++j) acc += g[j];
     }
     return acc;
 }
@@ -318,28 +324,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
         // (1) short rows: owner thread, CSR order; gathers issued before side effects
         if (v >= 0 && deg <= seq_max) {
             const double pv = pre(v);
-            double acc = 0.0;
-            const int e = beg + deg;
-            for (int a = beg; a < e; a += 4) {  // CSR order; +0.0 for padding slots
-                const bool v1 = a + 1 < e, v2 = a + 2 < e, v3 = a + 3 < e;
-                const int u0 = cols[a];
-                const int u1 = v1 ? cols[a + 1] : u0;
-                const int u2 = v2 ? cols[a + 2] : u0;
-                const int u3 = v3 ? cols[a + 3] : u0;
-                const int k0 = probe(u0), k1 = probe(u1), k2 = probe(u2), k3 = probe(u3);
-                const double g0 = gather(u0, k0);
-                const double g1 = v1 ? gather(u1, k1) : 0.0;
-                const double g2 = v2 ? gather(u2, k2) : 0.0;
-                const double g3 = v3 ? gather(u3, k3) : 0.0;
-                visit(u0, k0);
-                if (v1) visit(u1, k1);
-                if (v2) visit(u2, k2);
-                if (v3) visit(u3, k3);
-                acc += g0;
-                acc += g1;
-                acc += g2;
-                acc += g3;
-            }
+            const double acc = strided_sum<BC_UNROLL>(cols, beg, beg + deg, 1, probe, gather, visit);
             finish(v, acc, false, pv);
         }
         // (2) medium rows: the lanes of this warp take their rows one at a time
@@ -351,7 +336,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             const int b = __shfl_sync(FULL, beg, leader);
             const int e = b + __shfl_sync(FULL, deg, leader);
             const double pv = pre(w);
-            const double acc = warp_sum(coop_row(cols, b, e, lane, 32, probe, gather, visit));
+            const double acc = warp_sum(strided_sum<BC_UNROLL>(cols, b + lane, e, 32, probe, gather, visit));
             if (lane == leader) finish(w, acc, true, pv);
         }
         // (3) long rows: queued for the CTA-cooperative phase B
@@ -364,7 +349,8 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             const int v = __ldcg(&bigq[r]);
             const int b = rows[v], e = rows[v + 1];
             const double pv = pre(v);
-            const double acc = warp_sum(coop_row(cols, b, e, threadIdx.x, NT, probe, gather, visit));
+            const double acc =
+                warp_sum(strided_sum<BC_UNROLL>(cols, b + threadIdx.x, e, NT, probe, gather, visit));
             if (lane == 0) sm.red[wid] = acc;
             __syncthreads();
             if (threadIdx.x == 0) {
@@ -595,7 +581,10 @@ template <> __device__ __forceinline__ GlobalCodes make_levels<GlobalCodes>(cons
 // EPOK = false instantiates a work-efficient-only kernel (no EP code, fewer
 // registers) for launches that never run an EP level.
 template <bool DIR, class LV, int NT, bool EPOK>
-__global__ void __launch_bounds__(NT, NT >= 1024 ? 1 : (NT == 512 ? 2 : (NT == 256 ? 4 : 8)))
+#ifndef BC_MINB512
+#define BC_MINB512 2
+#endif
+__global__ void __launch_bounds__(NT, NT >= 1024 ? 1 : (NT == 512 ? BC_MINB512 : (NT == 256 ? 4 : 8)))
 bc_kernel(KParams p) {
     __shared__ Smem<NT> sm;
     extern __shared__ __align__(16) uint32_t dyn_smem[];
