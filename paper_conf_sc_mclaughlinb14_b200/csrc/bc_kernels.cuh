@@ -151,6 +151,7 @@ struct Smem {
 struct GlobalLevels {
     static constexpr int UNVISITED = INF;
     static constexpr bool RESET_VERTICES = true;
+    __device__ __forceinline__ void level_fence() const {}
     int *d;
     uint32_t *fb;  // unused
     __device__ __forceinline__ int probe(int u) const { return __ldcg(&d[u]); }
@@ -168,15 +169,22 @@ struct GlobalLevels {
 // 2-bit level codes in HBM/L2, per slot, for undirected graphs too large for
 // shared memory (n/4 bytes per source: 1 MB at n = 2^22, L2-resident for ~100
 // sources in flight instead of 16 MB of int32 distances).  Same code semantics
-// as SmemCodes; probes bypass L1 (ld.global.cg) because discoveries are atomics.
+// as SmemCodes; discoveries are global atomicOr.
 struct GlobalCodes {
     static constexpr int UNVISITED = 0;
     static constexpr bool RESET_VERTICES = false;
     uint32_t *w;
     uint32_t *fb;
+    // Probes go through L1 (neighbouring vertices share code words).  A stale L1
+    // line can only hide discoveries made by atomics; level_fence() invalidates L1
+    // (gpu-scope fence -> CCTL.IVALL) at every forward level start, so codes of
+    // earlier levels are always current.  Within a level a stale "unvisited" only
+    // costs a failed atomicOr (whose old value is authoritative); the backward
+    // stage performs no discoveries.
     __device__ __forceinline__ int probe(int u) const {
-        return (__ldcg(&w[u >> 4]) >> ((u & 15) << 1)) & 3;
+        return (__ldca(&w[u >> 4]) >> ((u & 15) << 1)) & 3;
     }
+    __device__ __forceinline__ void level_fence() const { __threadfence(); }
     __device__ __forceinline__ static int key(int L) { return L < 0 ? 4 : (L % 3) + 1; }
     __device__ __forceinline__ bool discover(int u, int L1) const {
         const uint32_t sh = (uint32_t)(u & 15) << 1;
@@ -210,6 +218,7 @@ struct GlobalCodes {
 struct SmemCodes {
     static constexpr int UNVISITED = 0;
     static constexpr bool RESET_VERTICES = false;
+    __device__ __forceinline__ void level_fence() const {}
     uint32_t *w;   // codes, 16 vertices per word
     uint32_t *fb;  // EP frontier bitmap, 32 vertices per word
     __device__ __forceinline__ int probe(int u) const { return (w[u >> 4] >> ((u & 15) << 1)) & 3; }
@@ -266,9 +275,9 @@ __device__ __forceinline__ double warp_sum(double v) {
 // (CSR order), stride = #cooperating threads for warp/CTA rows.  BC_UNROLL arcs
 // per step so that many col loads and gathers are in flight; padding slots add
 // +0.0, which leaves the CSR-order sum bit-identical.
-template <int U, class Probe, class Gather, class Visit>
+template <int U, class Probe, class Gather, class Claim, class Visit>
 __device__ __forceinline__ double strided_sum(const int *__restrict__ cols, int a, int e, int stride,
-                                              Probe &probe, Gather &gather, Visit &visit) {
+                                              Probe &probe, Gather &gather, Claim &claim, Visit &visit) {
     double acc = 0.0;
     for (; a < e; a += U * stride) {
         int u[U], k[U];
@@ -285,9 +294,12 @@ __device__ __forceinline__ double strided_sum(const int *__restrict__ cols, int 
         for (int j = 0; j < U; ++j) k[j] = probe(u[j]);
 #pragma unroll
         for (int j = 0; j < U; ++j) g[j] = ok[j] ? gather(u[j], k[j]) : 0.0;
+        bool won[U];  // all discovery atomics are issued before any result is used
+#pragma unroll
+        for (int j = 0; j < U; ++j) won[j] = ok[j] && claim(u[j], k[j]);
 #pragma unroll
         for (int j = 0; j < U; ++j)
-            if (ok[j]) visit(u[j], k[j]);
+            if (ok[j]) visit(u[j], k[j], won[j]);
 #pragma unroll
         for (int j = 0; j < U; ++j) acc += g[j];
     }
@@ -302,12 +314,12 @@ __device__ __forceinline__ double strided_sum(const int *__restrict__ cols, int 
 // thread in CSR order (the oracle's order); rows up to warp_max by one warp; longer
 // rows are queued in bigq and expanded by the whole CTA after one barrier.  Warps
 // take 32-vertex chunks independently, so there is no barrier per chunk.
-template <int NT, class Probe, class Gather, class Visit, class Pre, class Finish>
+template <int NT, class Probe, class Gather, class Claim, class Visit, class Pre, class Finish>
 __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int hi,
                                          const int *__restrict__ rows,
                                          const int *__restrict__ cols, int seq_max, int warp_max,
                                          int *__restrict__ bigq, Smem<NT> &sm, Counters &c,
-                                         Probe probe, Gather gather, Visit visit, Pre pre,
+                                         Probe probe, Gather gather, Claim claim, Visit visit, Pre pre,
                                          Finish finish) {
     constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -324,7 +336,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
         // (1) short rows: owner thread, CSR order; gathers issued before side effects
         if (v >= 0 && deg <= seq_max) {
             const double pv = pre(v);
-            const double acc = strided_sum<BC_UNROLL>(cols, beg, beg + deg, 1, probe, gather, visit);
+            const double acc = strided_sum<BC_UNROLL>(cols, beg, beg + deg, 1, probe, gather, claim, visit);
             finish(v, acc, false, pv);
         }
         // (2) medium rows: the lanes of this warp take their rows one at a time
@@ -336,7 +348,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             const int b = __shfl_sync(FULL, beg, leader);
             const int e = b + __shfl_sync(FULL, deg, leader);
             const double pv = pre(w);
-            const double acc = warp_sum(strided_sum<BC_UNROLL>(cols, b + lane, e, 32, probe, gather, visit));
+            const double acc = warp_sum(strided_sum<BC_UNROLL>(cols, b + lane, e, 32, probe, gather, claim, visit));
             if (lane == leader) finish(w, acc, true, pv);
         }
         // (3) long rows: queued for the CTA-cooperative phase B
@@ -350,7 +362,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             const int b = rows[v], e = rows[v + 1];
             const double pv = pre(v);
             const double acc =
-                warp_sum(strided_sum<BC_UNROLL>(cols, b + threadIdx.x, e, NT, probe, gather, visit));
+                warp_sum(strided_sum<BC_UNROLL>(cols, b + threadIdx.x, e, NT, probe, gather, claim, visit));
             if (lane == 0) sm.red[wid] = acc;
             __syncthreads();
             if (threadIdx.x == 0) {
@@ -390,8 +402,10 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
     const int kprev = LV::key(L - 1);
     auto probe = [&](int u) -> int { return lv.probe(u); };
     auto pull = [&](int u, int k) -> double { return k == kprev ? __ldcg(&sigma[u]) : 0.0; };
-    auto discover = [&](int u, int k) {
-        if (k == LV::UNVISITED && lv.discover(u, L1)) enqueue(S + hi, &sm.cnt[L % 3], u);
+    auto claim = [&](int u, int k) -> bool { return k == LV::UNVISITED && lv.discover(u, L1); };
+    auto noclaim = [&](int, int) -> bool { return false; };
+    auto discover = [&](int u, int, bool won) {
+        if (won) enqueue(S + hi, &sm.cnt[L % 3], u);
     };
     auto fin = [&](int v, double acc, bool coop, double) {
         sigma[v] = acc;
@@ -400,30 +414,30 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
     auto nopre = [&](int) -> double { return 0.0; };
     if (!DIR) {
         // fused: discovery of level L+1 and sigma pull for level L in one row scan
-        auto visit = [&](int u, int k) {
+        auto visit = [&](int u, int k, bool won) {
             if (k == kprev) c.dag++;
-            discover(u, k);
+            discover(u, k, won);
         };
         auto fin0 = [&](int v, double acc, bool coop, double) {
             if (L > 0) fin(v, acc, coop, 0.0);
         };
         const unsigned before = c.scanned;
         row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, pull,
-                     visit, nopre, fin0);
+                     claim, visit, nopre, fin0);
         c.arcs_reached += c.scanned - before;
     } else {
         auto none = [&](int, int) -> double { return 0.0; };
         auto fin1 = [&](int, double, bool, double) {};
         const unsigned before = c.scanned;
         row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, none,
-                     discover, nopre, fin1);
+                     claim, discover, nopre, fin1);
         c.arcs_reached += c.scanned - before;
         if (L > 0) {
-            auto count = [&](int, int k) {
+            auto count = [&](int, int k, bool) {
                 if (k == kprev) c.dag++;
             };
             row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe,
-                         pull, count, nopre, fin);
+                         pull, noclaim, count, nopre, fin);
         }
     }
 }
@@ -526,11 +540,12 @@ __device__ void backward_we(const KParams &p, const LV &lv, double *sig_om, cons
     const int knext = LV::key(L + 1);
     auto probe = [&](int v) -> int { return lv.probe(v); };
     auto gather = [&](int v, int k) -> double { return k == knext ? __ldcg(&sig_om[v]) : 0.0; };
-    auto none = [&](int, int) {};
+    auto noclaim = [&](int, int) -> bool { return false; };
+    auto none = [&](int, int, bool) {};
     auto pre = [&](int w) -> double { return __ldcg(&sig_om[w]); };  // sigma[w], issued early
     auto fin = [&](int w, double acc, bool, double sw) { finish_dependency(p, sw, sig_om, w, acc); };
-    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, gather, none,
-                 pre, fin);
+    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, gather,
+                 noclaim, none, pre, fin);
 }
 
 template <int NT, class LV>
@@ -584,7 +599,7 @@ template <bool DIR, class LV, int NT, bool EPOK>
 #ifndef BC_MINB512
 #define BC_MINB512 2
 #endif
-__global__ void __launch_bounds__(NT, NT >= 1024 ? 1 : (NT == 512 ? BC_MINB512 : (NT == 256 ? 4 : 8)))
+__global__ void __launch_bounds__(NT, NT >= 1024 ? 1 : (NT == 512 ? BC_MINB512 : (NT == 256 ? 4 : (NT == 128 ? 8 : 16))))
 bc_kernel(KParams p) {
     __shared__ Smem<NT> sm;
     extern __shared__ __align__(16) uint32_t dyn_smem[];
@@ -628,6 +643,7 @@ bc_kernel(KParams p) {
                                               : next_mode(p, MODE_WE, run_ep, 0, 1);
         for (;;) {
             const long long t0 = clock64();
+            lv.level_fence();
             if (!EPOK || mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             // (the level functions end with a barrier: every discovery is appended)

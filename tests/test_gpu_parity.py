@@ -353,3 +353,16 @@ def test_level_stores_agree(bcmod, oracle_mod, level_store, strategy):
             check_bc(bg, g, src, oracle_mod)
             s0 = int(src[0]) if src is not None else 7
             check_source(bg, g, s0, oracle_mod)
+
+
+@pytest.mark.parametrize("key", ["c5ws", "c5k"])
+def test_c5_subset_global_codes(bcmod, oracle_mod, key):
+    """Largest configs (n = 2^22, level codes in HBM/L2): BC over a seeded subset of the
+    config's sources and per-source d/sigma/delta against the oracle."""
+    g = graph(key)
+    src = gg.CONFIGS[key].sources(g)[:48]
+    with bcmod.BCGraph.from_graph(g) as bg:
+        assert bg.options()["strategy"] == bcmod.STRATEGIES["sampling"]
+        check_bc(bg, g, src, oracle_mod, nthreads=16)
+        for s in src[:2]:
+            check_source(bg, g, s, oracle_mod)
