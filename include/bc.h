@@ -82,6 +82,8 @@ typedef struct bc_options {
                                 by the whole CTA.  0 = auto (4096)                             */
     int32_t l2_persist;      /* 0 = auto (on), -1 = off: persisting-L2 access-policy window
                                 over the CSR arrays during traversal launches                  */
+    int32_t sort_frontier;   /* 0 = auto, 1 = on, -1 = off: rebuild large BFS levels in vertex
+                                order from a per-level bitmap (locality of rows, codes, sigma)  */
 } bc_options;
 
 typedef struct bc_stats {

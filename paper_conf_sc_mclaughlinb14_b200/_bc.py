@@ -31,7 +31,8 @@ class bc_options(ctypes.Structure):
                 ("ep_min_frontier", ctypes.c_int32), ("inflight", ctypes.c_int32),
                 ("backward_we", ctypes.c_int32), ("block_threads", ctypes.c_int32),
                 ("seq_max_deg", ctypes.c_int32), ("level_store", ctypes.c_int32),
-                ("warp_max_deg", ctypes.c_int32), ("l2_persist", ctypes.c_int32)]
+                ("warp_max_deg", ctypes.c_int32), ("l2_persist", ctypes.c_int32),
+                ("sort_frontier", ctypes.c_int32)]
 
 
 class bc_stats(ctypes.Structure):

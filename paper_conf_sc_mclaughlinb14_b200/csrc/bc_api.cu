@@ -67,6 +67,8 @@ struct bc_graph {
     } cfg_we, cfg_ep;
     int lstore = 1;       // level store: 1 int32 d (HBM), 2 codes in SMEM, 3 codes in HBM/L2
     uint32_t *gcodes = nullptr, *gfb = nullptr;
+    int sort_frontier = 0, sort_min = 0, nb_words = 0;  // sorted-frontier rebuild (configure())
+    uint32_t *nbits = nullptr;
     int code_words = 0, fb_words = 0;
     int seq_max_deg = 32;
     int warp_max_deg = 4096;
@@ -122,6 +124,7 @@ extern "C" void bc_default_options(bc_options *o) {
     o->seq_max_deg = 0;
     o->warp_max_deg = 0;
     o->l2_persist = 0;
+    o->sort_frontier = 0;
     o->level_store = 0;
 }
 
@@ -137,6 +140,8 @@ static void free_workspace(bc_graph *g) {
     cudaFree(g->bigq);
     cudaFree(g->gcodes);
     cudaFree(g->gfb);
+    cudaFree(g->nbits);
+    g->nbits = nullptr;
     g->bigq = nullptr;
     g->gcodes = g->gfb = nullptr;
     g->d = nullptr;
@@ -149,7 +154,8 @@ static void free_workspace(bc_graph *g) {
 static size_t slot_bytes(const bc_graph *g) {
     const size_t gc = g->lstore == 3 ? 4 * ((size_t)g->code_words + (size_t)g->fb_words) : 0;
     return g->stride_n * ((g->lstore == 1 ? sizeof(int) : 0) + 2 * sizeof(double) + sizeof(int)) +
-           g->stride_e * (sizeof(int) + 1) + g->stride_big * sizeof(int) + gc;
+           g->stride_e * (sizeof(int) + 1) + g->stride_big * sizeof(int) + gc +
+           (g->sort_frontier ? 4 * (size_t)g->nb_words : 0);
 }
 
 template <bool DIR, class LV, bool EPOK>
@@ -193,6 +199,12 @@ static int configure(bc_graph *g) {
         return fail(BC_EINVAL, "block_threads must be 0, 128, 256, 512 or 1024");
     g->seq_max_deg = o.seq_max_deg > 0 ? o.seq_max_deg : 32;
     g->warp_max_deg = std::max(g->seq_max_deg, o.warp_max_deg > 0 ? o.warp_max_deg : 4096);
+    // Sorted frontiers: a level is rebuilt in vertex order from the per-level bitmap
+    // when it holds >= sort_min vertices (the scan costs n/32 words, so small levels
+    // keep their append order).
+    g->sort_frontier = o.sort_frontier > 0 ? 1 : (o.sort_frontier < 0 ? 0 : (g->n >= (1 << 17)));
+    g->nb_words = (int)((((size_t)g->n + 31) / 32 + 31) & ~(size_t)31);
+    g->sort_min = std::max(1024, g->n / 64);
     g->code_words = g->lstore >= 2 ? (int)(code_bytes / 4) : 0;
     g->fb_words = g->lstore >= 2 ? (int)(fb_bytes / 4) : 0;
 
@@ -259,6 +271,10 @@ static int alloc_workspace(bc_graph *g) {
     CK(cudaMalloc(&g->ends, ns * g->stride_e * sizeof(int)));
     CK(cudaMalloc(&g->modes, ns * g->stride_e));
     CK(cudaMalloc(&g->bigq, ns * g->stride_big * sizeof(int)));
+    if (g->sort_frontier) {
+        CK(cudaMalloc(&g->nbits, ns * (size_t)g->nb_words * 4));
+        CK(cudaMemset(g->nbits, 0, ns * (size_t)g->nb_words * 4));
+    }
     if (g->lstore == 1) CK(cudaMemset(g->d, 0x7F, ns * g->stride_n * sizeof(int)));  // INF = 0x7F7F7F7F
     CK(cudaMemset(g->sigma, 0, ns * g->stride_n * sizeof(double)));
     CK(cudaMemset(g->omega, 0, ns * g->stride_n * sizeof(double)));
@@ -454,7 +470,8 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     }
     const int old_slots = g->slots;
     const int realloc = o->inflight != old.inflight || o->level_store != old.level_store ||
-                        o->block_threads != old.block_threads || o->warp_max_deg != old.warp_max_deg;
+                        o->block_threads != old.block_threads || o->warp_max_deg != old.warp_max_deg ||
+                        o->sort_frontier != old.sort_frontier;
     if (realloc) {
         rc = alloc_workspace(g);
         if (rc) return rc;
@@ -500,6 +517,10 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     p.gfb = g->gfb;
     p.stride_codes = (size_t)g->code_words;
     p.stride_fb = (size_t)g->fb_words;
+    p.nbits = g->sort_frontier ? g->nbits : nullptr;
+    p.stride_nb = (size_t)g->nb_words;
+    p.nb_words = g->nb_words;
+    p.sort_min = g->sort_min;
     p.seq_max_deg = g->seq_max_deg;
     p.warp_max_deg = g->warp_max_deg;
     p.stats = g->stats;

@@ -82,6 +82,10 @@ struct KParams {
     uint32_t *gfb;
     size_t stride_codes, stride_fb;
     int fb_words;        // 0: this launch never runs an EP level
+    uint32_t *nbits;     // per-slot bitmap of the level being discovered (sorted frontiers)
+    size_t stride_nb;
+    int nb_words;
+    int sort_min;        // rebuild a level in vertex order when it has >= sort_min vertices
     int seq_max_deg;     // rows up to this degree: owner thread, CSR order
     int warp_max_deg;    // rows up to this degree: one warp; longer: whole CTA
     // strategy
@@ -140,6 +144,7 @@ struct Smem {
     int nbig;             // rows queued for CTA-cooperative expansion in this tile
     CtaStats st;
     double red[NT / 32];  // block reduction scratch
+    int wtot[NT / 32];    // per-warp totals (frontier compaction)
     int big_v[NT];
     int big_beg[NT];
     int big_deg[NT];
@@ -393,11 +398,52 @@ __device__ __forceinline__ int next_mode(const KParams &p, int mode, int run_ep,
     }
 }
 
+// Rewrite out[0 .. popcount(nb)) with the set bits of nb in ascending order and
+// clear nb.  Each warp owns a contiguous range of words and reads it coalesced;
+// one block scan of the warp totals.  Ends with a barrier.
+template <int NT>
+__device__ __forceinline__ void compact_level(uint32_t *nb, int words, int *out, Smem<NT> &sm) {
+    constexpr int NW = NT / 32;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int per = ((words + NW - 1) / NW + 31) & ~31;  // words per warp, multiple of 32
+    const int w0 = min(wid * per, words), w1 = min(w0 + per, words);
+    int cnt = 0;
+    for (int w = w0 + lane; w < w1; w += 32) cnt += __popc(__ldcg(&nb[w]));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
+    if (lane == 0) sm.wtot[wid] = cnt;
+    __syncthreads();
+    int base = 0;
+    for (int q = 0; q < wid; ++q) base += sm.wtot[q];
+    for (int w = w0; w < w1; w += 32) {
+        const int wi = w + lane;
+        uint32_t bits = wi < w1 ? __ldcg(&nb[wi]) : 0u;
+        const int c = __popc(bits);
+        int incl = c;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += y;
+        }
+        int pos = base + incl - c;
+        if (bits) {
+            nb[wi] = 0u;
+            while (bits) {
+                const int b = __ffs(bits) - 1;
+                out[pos++] = wi * 32 + b;
+                bits &= bits - 1u;
+            }
+        }
+        base += __shfl_sync(FULL, incl, 31);
+    }
+    __syncthreads();
+}
+
 // ------------------------------------------------------------------ forward
 
 template <bool DIR, int NT, class LV>
-__device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S, int *bigq, int L,
-                           int lo, int hi, Smem<NT> &sm, Counters &c) {
+__device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S, int *bigq,
+                           uint32_t *nb, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int L1 = L + 1;
     const int kprev = LV::key(L - 1);
     auto probe = [&](int u) -> int { return lv.probe(u); };
@@ -405,7 +451,10 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
     auto claim = [&](int u, int k) -> bool { return k == LV::UNVISITED && lv.discover(u, L1); };
     auto noclaim = [&](int, int) -> bool { return false; };
     auto discover = [&](int u, int, bool won) {
-        if (won) enqueue(S + hi, &sm.cnt[L % 3], u);
+        if (won) {
+            enqueue(S + hi, &sm.cnt[L % 3], u);
+            if (nb) atomicOr(&nb[u >> 5], 1u << (u & 31));  // RED: result unused
+        }
     };
     auto fin = [&](int v, double acc, bool coop, double) {
         sigma[v] = acc;
@@ -611,6 +660,7 @@ bc_kernel(KParams p) {
     int *ends = p.ends + slot * p.stride_e;
     unsigned char *modes = p.modes + slot * p.stride_e;
     int *bigq = p.bigq + slot * p.stride_big;
+    uint32_t *nb = p.nbits ? p.nbits + slot * p.stride_nb : nullptr;
 
     Counters c;
     const int run_ep = (p.launch_mode == LM_SAMPLED && p.sampled_flag) ? *p.sampled_flag : 0;
@@ -644,7 +694,10 @@ bc_kernel(KParams p) {
         for (;;) {
             const long long t0 = clock64();
             lv.level_fence();
-            if (!EPOK || mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, L, lo, hi, sm, c);
+            // mark discoveries in the bitmap only when the next level is likely to be
+            // large enough to be rebuilt (levels grow/shrink gradually)
+            uint32_t *const nbl = (nb && (long long)(hi - lo) * 4 >= p.sort_min) ? nb : nullptr;
+            if (!EPOK || mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, nbl, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             // (the level functions end with a barrier: every discovery is appended)
             const int nhi = hi + sm.cnt[L % 3];
@@ -656,6 +709,16 @@ bc_kernel(KParams p) {
                 sm.cnt[(L + 2) % 3] = 0;
                 sm.st.cyc[mode] += (unsigned long long)(clock64() - t0);
                 sm.st.lv[mode] += 1;
+            }
+            if (nbl && mode == MODE_WE && nhi > hi) {
+                // Level L+1 in vertex order (any order is a valid S, R14): consecutive
+                // threads then touch neighbouring rows, codes and sigma entries.
+                if (nhi - hi >= p.sort_min) {
+                    compact_level<NT>(nb, p.nb_words, S + hi, sm);
+                } else {
+                    for (int i = hi + threadIdx.x; i < nhi; i += NT) nb[S[i] >> 5] = 0u;
+                    __syncthreads();
+                }
             }
             if (nhi == hi) break;  // Q_next_len == 0 (Alg. 2 l.11)
             mode = next_mode(p, mode, run_ep, hi - lo, nhi - hi);

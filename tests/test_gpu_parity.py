@@ -366,3 +366,15 @@ def test_c5_subset_global_codes(bcmod, oracle_mod, key):
         check_bc(bg, g, src, oracle_mod, nthreads=16)
         for s in src[:2]:
             check_source(bg, g, s, oracle_mod)
+
+
+@pytest.mark.parametrize("sort_frontier", [-1, 1])
+def test_sorted_frontier_rebuild(bcmod, oracle_mod, sort_frontier):
+    """Levels rebuilt in vertex order from the discovery bitmap (any order of S within a
+    level is valid, R14) give identical d/sigma and BC within tolerance."""
+    for key, k in (("c1", None), ("c3", 200), ("c4", 200)):
+        g = graph(key)
+        src = None if k is None else gg.CONFIGS[key].sources(g)[:k]
+        with bcmod.BCGraph.from_graph(g, strategy="we", sort_frontier=sort_frontier) as bg:
+            check_bc(bg, g, src, oracle_mod)
+            check_source(bg, g, 5 if src is None else int(src[1]), oracle_mod)
