@@ -203,6 +203,7 @@ static int configure(bc_graph *g) {
     // when it holds >= sort_min vertices (the scan costs n/32 words, so small levels
     // keep their append order).
     g->sort_frontier = o.sort_frontier > 0 ? 1 : (o.sort_frontier < 0 ? 0 : (g->n >= (1 << 17)));
+    if (g->lstore == 3) g->sort_frontier = 1;  // codes in HBM/L2 discover through the bitmap
     g->nb_words = (int)((((size_t)g->n + 31) / 32 + 31) & ~(size_t)31);
     g->sort_min = std::max(1024, g->n / 64);
     g->code_words = g->lstore >= 2 ? (int)(code_bytes / 4) : 0;

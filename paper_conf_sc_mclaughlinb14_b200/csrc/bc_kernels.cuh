@@ -156,6 +156,8 @@ struct Smem {
 struct GlobalLevels {
     static constexpr int UNVISITED = INF;
     static constexpr bool RESET_VERTICES = true;
+    static constexpr bool BITMAP_DISCOVERY = false;
+    __device__ __forceinline__ void mark(int, int) const {}
     __device__ __forceinline__ void level_fence() const {}
     int *d;
     uint32_t *fb;  // unused
@@ -178,6 +180,12 @@ struct GlobalLevels {
 struct GlobalCodes {
     static constexpr int UNVISITED = 0;
     static constexpr bool RESET_VERTICES = false;
+    // Discovery without winner election: mark() is an idempotent OR (RED, no return)
+    // and the level is rebuilt from the per-level bitmap (compact_level).
+    static constexpr bool BITMAP_DISCOVERY = true;
+    __device__ __forceinline__ void mark(int u, int L1) const {
+        atomicOr(&w[u >> 4], (uint32_t)key(L1) << ((u & 15) << 1));
+    }
     uint32_t *w;
     uint32_t *fb;
     // Probes go through L1 (neighbouring vertices share code words).  A stale L1
@@ -223,6 +231,8 @@ struct GlobalCodes {
 struct SmemCodes {
     static constexpr int UNVISITED = 0;
     static constexpr bool RESET_VERTICES = false;
+    static constexpr bool BITMAP_DISCOVERY = false;
+    __device__ __forceinline__ void mark(int, int) const {}
     __device__ __forceinline__ void level_fence() const {}
     uint32_t *w;   // codes, 16 vertices per word
     uint32_t *fb;  // EP frontier bitmap, 32 vertices per word
@@ -400,9 +410,9 @@ __device__ __forceinline__ int next_mode(const KParams &p, int mode, int run_ep,
 
 // Rewrite out[0 .. popcount(nb)) with the set bits of nb in ascending order and
 // clear nb.  Each warp owns a contiguous range of words and reads it coalesced;
-// one block scan of the warp totals.  Ends with a barrier.
+// one block scan of the warp totals.  Returns popcount(nb); ends with a barrier.
 template <int NT>
-__device__ __forceinline__ void compact_level(uint32_t *nb, int words, int *out, Smem<NT> &sm) {
+__device__ __forceinline__ int compact_level(uint32_t *nb, int words, int *out, Smem<NT> &sm) {
     constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int per = ((words + NW - 1) / NW + 31) & ~31;  // words per warp, multiple of 32
@@ -413,8 +423,11 @@ __device__ __forceinline__ void compact_level(uint32_t *nb, int words, int *out,
     for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
     if (lane == 0) sm.wtot[wid] = cnt;
     __syncthreads();
-    int base = 0;
-    for (int q = 0; q < wid; ++q) base += sm.wtot[q];
+    int base = 0, total = 0;
+    for (int q = 0; q < NW; ++q) {
+        if (q < wid) base += sm.wtot[q];
+        total += sm.wtot[q];
+    }
     for (int w = w0; w < w1; w += 32) {
         const int wi = w + lane;
         uint32_t bits = wi < w1 ? __ldcg(&nb[wi]) : 0u;
@@ -437,6 +450,7 @@ __device__ __forceinline__ void compact_level(uint32_t *nb, int words, int *out,
         base += __shfl_sync(FULL, incl, 31);
     }
     __syncthreads();
+    return total;
 }
 
 // ------------------------------------------------------------------ forward
@@ -448,7 +462,18 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
     const int kprev = LV::key(L - 1);
     auto probe = [&](int u) -> int { return lv.probe(u); };
     auto pull = [&](int u, int k) -> double { return k == kprev ? __ldcg(&sigma[u]) : 0.0; };
-    auto claim = [&](int u, int k) -> bool { return k == LV::UNVISITED && lv.discover(u, L1); };
+    auto claim = [&](int u, int k) -> bool {
+        if (LV::BITMAP_DISCOVERY) {
+            // no winner election: idempotent OR of the code and of the level bitmap
+            // (fire-and-forget RED); the level is compacted from the bitmap afterwards
+            if (k == LV::UNVISITED) {
+                lv.mark(u, L1);
+                atomicOr(&nb[u >> 5], 1u << (u & 31));
+            }
+            return false;
+        }
+        return k == LV::UNVISITED && lv.discover(u, L1);
+    };
     auto noclaim = [&](int, int) -> bool { return false; };
     auto discover = [&](int u, int, bool won) {
         if (won) {
@@ -696,11 +721,29 @@ bc_kernel(KParams p) {
             lv.level_fence();
             // mark discoveries in the bitmap only when the next level is likely to be
             // large enough to be rebuilt (levels grow/shrink gradually)
-            uint32_t *const nbl = (nb && (long long)(hi - lo) * 4 >= p.sort_min) ? nb : nullptr;
+            uint32_t *const nbl =
+                LV::BITMAP_DISCOVERY ? nb
+                                     : ((nb && (long long)(hi - lo) * 4 >= p.sort_min) ? nb : nullptr);
             if (!EPOK || mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, nbl, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
-            // (the level functions end with a barrier: every discovery is appended)
-            const int nhi = hi + sm.cnt[L % 3];
+            // (the level functions end with a barrier: every discovery is recorded)
+            int nhi;
+            if (LV::BITMAP_DISCOVERY && mode == MODE_WE) {
+                // level L+1 = the discovery bitmap, written to S in vertex order
+                nhi = hi + compact_level<NT>(nb, p.nb_words, S + hi, sm);
+            } else {
+                nhi = hi + sm.cnt[L % 3];
+                if (nbl && mode == MODE_WE && nhi > hi) {
+                    // Level L+1 in vertex order (any order is a valid S, R14): consecutive
+                    // threads then touch neighbouring rows, codes and sigma entries.
+                    if (nhi - hi >= p.sort_min) {
+                        compact_level<NT>(nb, p.nb_words, S + hi, sm);
+                    } else {
+                        for (int i = hi + threadIdx.x; i < nhi; i += NT) nb[S[i] >> 5] = 0u;
+                        __syncthreads();
+                    }
+                }
+            }
             if (threadIdx.x == 0) {
                 modes[L] = (unsigned char)mode;
                 ends[L + 2] = nhi;
@@ -709,16 +752,6 @@ bc_kernel(KParams p) {
                 sm.cnt[(L + 2) % 3] = 0;
                 sm.st.cyc[mode] += (unsigned long long)(clock64() - t0);
                 sm.st.lv[mode] += 1;
-            }
-            if (nbl && mode == MODE_WE && nhi > hi) {
-                // Level L+1 in vertex order (any order is a valid S, R14): consecutive
-                // threads then touch neighbouring rows, codes and sigma entries.
-                if (nhi - hi >= p.sort_min) {
-                    compact_level<NT>(nb, p.nb_words, S + hi, sm);
-                } else {
-                    for (int i = hi + threadIdx.x; i < nhi; i += NT) nb[S[i] >> 5] = 0u;
-                    __syncthreads();
-                }
             }
             if (nhi == hi) break;  // Q_next_len == 0 (Alg. 2 l.11)
             mode = next_mode(p, mode, run_ep, hi - lo, nhi - hi);
