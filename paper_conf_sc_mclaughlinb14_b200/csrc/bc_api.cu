@@ -385,7 +385,7 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col_in) 
         for (int u = 0; u < n; ++u)
             for (int e = ro32[u]; e < ro32[u + 1]; ++e) icol[fill[col[e]]++] = u;
         CK(cudaMalloc(&g->iro, sizeof(int) * ((size_t)n + 1)));
-        CK(cudaMalloc(&g->icol, sizeof(int) * (size_t)std::max(nnz, 1)));
+        CK(cudaMalloc(&g->icol, sizeof(int) * ((size_t)std::max(nnz, 1) + 4)));  // quad-read slack
         CK(cudaMalloc(&g->isrc, sizeof(int) * (size_t)std::max(nnz, 1)));
         CK(cudaMemcpy(g->iro, iro.data(), sizeof(int) * ((size_t)n + 1), cudaMemcpyHostToDevice));
         if (nnz) {
