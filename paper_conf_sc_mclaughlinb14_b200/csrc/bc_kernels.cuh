@@ -294,16 +294,24 @@ template <int U, class Probe, class Gather, class Claim, class Visit>
 __device__ __forceinline__ double strided_sum(const int *__restrict__ cols, int a, int e, int stride,
                                               Probe &probe, Gather &gather, Claim &claim, Visit &visit) {
     double acc = 0.0;
+    // software pipeline: the col loads of step i+1 are issued before the gathers of
+    // step i are consumed (padding slots probe vertex 0 and add +0.0)
+    int un[U];
+#pragma unroll
+    for (int j = 0; j < U; ++j) un[j] = a + j * stride < e ? cols[a + j * stride] : 0;
     for (; a < e; a += U * stride) {
         int u[U], k[U];
         bool ok[U];
         double g[U];
-        u[0] = cols[a];
-        ok[0] = true;
 #pragma unroll
-        for (int j = 1; j < U; ++j) {
+        for (int j = 0; j < U; ++j) {
+            u[j] = un[j];
             ok[j] = a + j * stride < e;
-            u[j] = ok[j] ? cols[a + j * stride] : u[0];
+        }
+        const int an = a + U * stride;
+        if (an < e) {
+#pragma unroll
+            for (int j = 0; j < U; ++j) un[j] = an + j * stride < e ? cols[an + j * stride] : 0;
         }
 #pragma unroll
         for (int j = 0; j < U; ++j) k[j] = probe(u[j]);
