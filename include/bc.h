@@ -84,6 +84,11 @@ typedef struct bc_options {
                                 over the CSR arrays during traversal launches                  */
     int32_t sort_frontier;   /* 0 = auto, 1 = on, -1 = off: rebuild large BFS levels in vertex
                                 order from a per-level bitmap (locality of rows, codes, sigma)  */
+    /* Output post-processing (default 0 = exact BC as defined above): */
+    int32_t extrapolate;     /* 1: multiply by n/k (k = number of sources): the k-source
+                                estimator of total BC ("trivially adjusted for approximation",
+                                P:315, refs [3],[9])                                            */
+    int32_t normalize;       /* 1: divide by (n-1)(n-2), the normalisation of P:74             */
 } bc_options;
 
 typedef struct bc_stats {
@@ -145,6 +150,16 @@ BC_API int bc_compute_device(bc_graph *g, const int32_t *d_sources, int64_t k, d
  *   num_levels   receives maxdepth + 1 */
 BC_API int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigma, double *delta,
                      uint8_t *level_modes, int32_t max_levels, int32_t *num_levels);
+
+/* Per-level trace of one source (the paper's Table I / Fig. 3 study,
+ * P:231-263), computed exactly like bc_single_source with one CTA:
+ *   level_sizes  int32[max_levels]  vertex frontier |{v : d(s,v) = L}| per level L
+ *   fwd_cycles   int64[max_levels]  SM cycles spent on forward level L (incl. bookkeeping)
+ *   bwd_cycles   int64[max_levels]  SM cycles spent on backward level L (0 for L = 0 and the
+ *                                   deepest level, which Alg. 3 does not process)
+ *   num_levels   receives maxdepth + 1 (arrays hold min(max_levels, num_levels) entries) */
+BC_API int bc_trace_source(bc_graph *g, int32_t s, int32_t *level_sizes, int64_t *fwd_cycles,
+                           int64_t *bwd_cycles, int32_t max_levels, int32_t *num_levels);
 
 BC_API void bc_default_options(bc_options *o);
 BC_API int bc_set_options(bc_graph *g, const bc_options *o); /* validates; may reallocate workspace */

@@ -21,8 +21,8 @@ BC_STRATEGY_WE, BC_STRATEGY_EP, BC_STRATEGY_HYBRID, BC_STRATEGY_SAMPLING = 0, 1,
 STRATEGIES = {"we": 0, "ep": 1, "hybrid": 2, "sampling": 3}
 
 EXPORTED = ("bc_graph_create", "bc_compute", "bc_compute_device", "bc_single_source",
-            "bc_default_options", "bc_set_options", "bc_get_options", "bc_get_stats",
-            "bc_destroy", "bc_last_error")
+            "bc_trace_source", "bc_default_options", "bc_set_options", "bc_get_options",
+            "bc_get_stats", "bc_destroy", "bc_last_error")
 
 
 class bc_options(ctypes.Structure):
@@ -32,7 +32,8 @@ class bc_options(ctypes.Structure):
                 ("backward_we", ctypes.c_int32), ("block_threads", ctypes.c_int32),
                 ("seq_max_deg", ctypes.c_int32), ("level_store", ctypes.c_int32),
                 ("warp_max_deg", ctypes.c_int32), ("l2_persist", ctypes.c_int32),
-                ("sort_frontier", ctypes.c_int32)]
+                ("sort_frontier", ctypes.c_int32), ("extrapolate", ctypes.c_int32),
+                ("normalize", ctypes.c_int32)]
 
 
 class bc_stats(ctypes.Structure):
@@ -80,6 +81,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.bc_compute_device.argtypes = [_vp, _vp, ctypes.c_int64, _vp, _vp]
     lib.bc_single_source.argtypes = [_vp, ctypes.c_int32, _i32p, _f64p, _f64p, _u8p,
                                      ctypes.c_int32, _i32p]
+    lib.bc_trace_source.argtypes = [_vp, ctypes.c_int32, _i32p, _i64p, _i64p, ctypes.c_int32, _i32p]
     lib.bc_default_options.argtypes = [ctypes.POINTER(bc_options)]
     lib.bc_default_options.restype = None
     lib.bc_set_options.argtypes = [_vp, ctypes.POINTER(bc_options)]
@@ -90,7 +92,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.bc_last_error.argtypes = []
     lib.bc_last_error.restype = ctypes.c_char_p
     for name in ("bc_graph_create", "bc_compute", "bc_compute_device", "bc_single_source",
-                 "bc_set_options", "bc_get_options", "bc_get_stats"):
+                 "bc_trace_source", "bc_set_options", "bc_get_options", "bc_get_stats"):
         getattr(lib, name).restype = ctypes.c_int
     _lib = lib
     return lib
@@ -155,6 +157,20 @@ def bc_single_source(handle: int, n: int, s: int, max_levels: Optional[int] = No
                                 _ptr(delta, _f64p), _ptr(modes, _u8p), int(ml), ctypes.byref(nl)))
     L = nl.value
     return dict(d=d, sigma=sigma, delta=delta, level_modes=modes[:min(L, ml)].copy(), num_levels=L)
+
+
+def bc_trace_source(handle: int, s: int, max_levels: int = 1 << 16) -> dict:
+    """Per-level frontier sizes and forward/backward SM cycles of one source (N2)."""
+    lib = load_library()
+    ls = np.zeros(max_levels, dtype=np.int32)
+    fc = np.zeros(max_levels, dtype=np.int64)
+    bcyc = np.zeros(max_levels, dtype=np.int64)
+    nl = ctypes.c_int32(0)
+    _check(lib.bc_trace_source(_vp(handle), int(s), _ptr(ls, _i32p), _ptr(fc, _i64p),
+                               _ptr(bcyc, _i64p), int(max_levels), ctypes.byref(nl)))
+    L = min(nl.value, max_levels)
+    return dict(level_sizes=ls[:L].copy(), fwd_cycles=fc[:L].copy(), bwd_cycles=bcyc[:L].copy(),
+                num_levels=nl.value)
 
 
 def bc_default_options() -> bc_options:
@@ -231,6 +247,9 @@ class BCGraph:
 
     def single_source(self, s: int, max_levels: Optional[int] = None) -> dict:
         return bc_single_source(self.handle, self.n, s, max_levels)
+
+    def trace_source(self, s: int, max_levels: int = 1 << 16) -> dict:
+        return bc_trace_source(self.handle, s, max_levels)
 
     def stats(self) -> dict:
         return bc_get_stats(self.handle)

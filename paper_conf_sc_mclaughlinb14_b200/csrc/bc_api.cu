@@ -125,6 +125,8 @@ extern "C" void bc_default_options(bc_options *o) {
     o->warp_max_deg = 0;
     o->l2_persist = 0;
     o->sort_frontier = 0;
+    o->extrapolate = 0;
+    o->normalize = 0;
     o->level_store = 0;
 }
 
@@ -635,13 +637,17 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
             g->tev_used[1] = 1;
         }
     }
-    const double h = g->directed ? 1.0 : 0.5;
+    double h = g->directed ? 1.0 : 0.5;
+    // optional k-source estimator scaling (n/k, refs [3],[9]) and the
+    // (n-1)(n-2) normalisation of P:74 (applied literally as written in the paper).
+    if (g->opt.extrapolate && k > 0) h *= (double)g->n / (double)k;
+    if (g->opt.normalize && g->n > 2) h /= ((double)g->n - 1.0) * ((double)g->n - 2.0);
     const int eb = std::min((g->n + 255) / 256, 148 * 8);
     if (g->perm) {
         unpermute_kernel<<<eb, 256, 0, st>>>(acc_bc, g->perm, g->n, h, d_bc);
         CK(cudaGetLastError());
         g->launches++;
-    } else if (!g->directed) {
+    } else if (h != 1.0) {
         scale_kernel<<<eb, 256, 0, st>>>(d_bc, g->n, h);
         CK(cudaGetLastError());
         g->launches++;
@@ -690,21 +696,31 @@ extern "C" int bc_compute(bc_graph *g, const int32_t *sources, int64_t num_sourc
     return BC_OK;
 }
 
-extern "C" int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigma, double *delta,
-                                uint8_t *level_modes, int32_t max_levels, int32_t *num_levels) {
+static int single_source_impl(bc_graph *g, int32_t s, int32_t *d, double *sigma, double *delta,
+                              uint8_t *level_modes, int32_t max_levels, int32_t *num_levels,
+                              int32_t *level_sizes, int64_t *fwd_cycles, int64_t *bwd_cycles) {
     if (!g) return fail(BC_EINVAL, "NULL graph");
     if (s < 0 || s >= g->n) return fail(BC_EINVAL, "source %d out of range", s);
-    if (level_modes && max_levels < 0) return fail(BC_EINVAL, "max_levels < 0");
+    if (max_levels < 0) return fail(BC_EINVAL, "max_levels < 0");
     DeviceGuard dg(g->device);
     CK(cudaEventSynchronize(g->done));
     const size_t n = (size_t)g->n;
-    const int ml = level_modes ? max_levels : 0;
-    int *dd = nullptr, *dn = nullptr, *dsrc = nullptr;
+    const bool trace = level_sizes || fwd_cycles || bwd_cycles;
+    const int ml = (level_modes || trace) ? max_levels : 0;
+    int *dd = nullptr, *dn = nullptr, *dsrc = nullptr, *dls = nullptr;
     double *ds = nullptr, *ddel = nullptr, *dbc = nullptr;
+    long long *dfc = nullptr, *dbcyc = nullptr;
     unsigned char *dm = nullptr;
     int rc = BC_OK;
     cudaError_t e = cudaSuccess;
-    e = cudaMalloc(&dd, n * sizeof(int));
+    if (trace) {
+        const size_t lv = (size_t)std::max(ml, 1);
+        e = cudaMalloc(&dls, lv * sizeof(int));
+        if (e == cudaSuccess) e = cudaMalloc(&dfc, lv * sizeof(long long));
+        if (e == cudaSuccess) e = cudaMalloc(&dbcyc, lv * sizeof(long long));
+        if (e == cudaSuccess) e = cudaMemsetAsync(dbcyc, 0, lv * sizeof(long long), g->stream);
+    }
+    if (e == cudaSuccess) e = cudaMalloc(&dd, n * sizeof(int));
     if (e == cudaSuccess) e = cudaMalloc(&ds, n * sizeof(double));
     if (e == cudaSuccess) e = cudaMalloc(&ddel, n * sizeof(double));
     if (e == cudaSuccess) e = cudaMalloc(&dbc, n * sizeof(double));
@@ -737,6 +753,9 @@ extern "C" int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigm
         p.dbg_modes = dm;
         p.dbg_max_levels = ml;
         p.dbg_nlevels = dn;
+        p.dbg_lsizes = dls;
+        p.dbg_fcyc = dfc;
+        p.dbg_bcyc = dbcyc;
         p.stats = dst;  // keep the last compute call's stats intact
         rc = launch(g, p, g->stream);
     }
@@ -759,11 +778,21 @@ extern "C" int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigm
         if (e == cudaSuccess) e = fetch(sigma, ds, sizeof(double));
         if (e == cudaSuccess) e = fetch(delta, ddel, sizeof(double));
         if (e == cudaSuccess) e = cudaMemcpy(&nl, dn, sizeof(int), cudaMemcpyDeviceToHost);
-        if (e == cudaSuccess && level_modes && ml > 0)
-            e = cudaMemcpy(level_modes, dm, (size_t)std::min(ml, nl), cudaMemcpyDeviceToHost);
+        const size_t nlc = (size_t)std::max(0, std::min(ml, nl));
+        if (e == cudaSuccess && level_modes && nlc)
+            e = cudaMemcpy(level_modes, dm, nlc, cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess && level_sizes && nlc)
+            e = cudaMemcpy(level_sizes, dls, nlc * sizeof(int), cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess && fwd_cycles && nlc)
+            e = cudaMemcpy(fwd_cycles, dfc, nlc * sizeof(long long), cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess && bwd_cycles && nlc)
+            e = cudaMemcpy(bwd_cycles, dbcyc, nlc * sizeof(long long), cudaMemcpyDeviceToHost);
         if (e != cudaSuccess) rc = fail(BC_ECUDA, "%s", cudaGetErrorString(e));
     }
     if (rc == BC_OK && num_levels) *num_levels = nl;
+    cudaFree(dls);
+    cudaFree(dfc);
+    cudaFree(dbcyc);
     cudaFree(dd);
     cudaFree(ds);
     cudaFree(ddel);
@@ -774,6 +803,19 @@ extern "C" int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigm
     cudaFree(dst);
     if (rc == BC_OK) g_err[0] = 0;
     return rc;
+}
+
+extern "C" int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigma, double *delta,
+                                uint8_t *level_modes, int32_t max_levels, int32_t *num_levels) {
+    return single_source_impl(g, s, d, sigma, delta, level_modes, level_modes ? max_levels : 0,
+                              num_levels, nullptr, nullptr, nullptr);
+}
+
+extern "C" int bc_trace_source(bc_graph *g, int32_t s, int32_t *level_sizes, int64_t *fwd_cycles,
+                               int64_t *bwd_cycles, int32_t max_levels, int32_t *num_levels) {
+    if (!level_sizes || !fwd_cycles || !bwd_cycles) return fail(BC_EINVAL, "NULL trace array");
+    return single_source_impl(g, s, nullptr, nullptr, nullptr, nullptr, max_levels, num_levels,
+                              level_sizes, fwd_cycles, bwd_cycles);
 }
 
 extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {

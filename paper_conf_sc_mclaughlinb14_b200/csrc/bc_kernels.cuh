@@ -102,6 +102,10 @@ struct KParams {
     unsigned char *dbg_modes;
     int dbg_max_levels;
     int *dbg_nlevels;
+    // per-level trace, may be NULL: frontier sizes and SM cycles
+    int *dbg_lsizes;
+    long long *dbg_fcyc;
+    long long *dbg_bcyc;
 };
 
 // Per-thread counters for the byte model / stats, flushed into shared memory once
@@ -792,7 +796,9 @@ bc_kernel(KParams p) {
                 // cnt[(L+2)%3] was last used by level L-1 and read by every thread
                 // before level L started; it is next used by level L+2.
                 sm.cnt[(L + 2) % 3] = 0;
-                sm.st.cyc[mode] += (unsigned long long)(clock64() - t0);
+                const long long dt = clock64() - t0;
+                sm.st.cyc[mode] += (unsigned long long)dt;
+                if (p.dbg_fcyc && L < p.dbg_max_levels) p.dbg_fcyc[L] = dt;
                 sm.st.lv[mode] += 1;
             }
             if (nhi == hi) break;  // Q_next_len == 0 (Alg. 2 l.11)
@@ -826,13 +832,20 @@ bc_kernel(KParams p) {
             const long long t0 = clock64();
             if (!EPOK || bmode == MODE_WE) backward_we<NT>(p, lv, sigma, S, bigq, Lb, blo, bhi, sm, c);
             else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
-            if (threadIdx.x == 0) sm.st.cyc[2 + bmode] += (unsigned long long)(clock64() - t0);
+            if (threadIdx.x == 0) {
+                const long long dt = clock64() - t0;
+                sm.st.cyc[2 + bmode] += (unsigned long long)dt;
+                if (p.dbg_bcyc && Lb < p.dbg_max_levels) p.dbg_bcyc[Lb] = dt;
+            }
         }
 
         // Debug export, then reset of the touched state.
         if (p.dbg_d) {
             if (threadIdx.x == 0) {
-                for (int l = 0; l <= maxdepth && l < p.dbg_max_levels; ++l) p.dbg_modes[l] = modes[l];
+                for (int l = 0; l <= maxdepth && l < p.dbg_max_levels; ++l) {
+                    p.dbg_modes[l] = modes[l];
+                    if (p.dbg_lsizes) p.dbg_lsizes[l] = ends[l + 1] - ends[l];
+                }
                 *p.dbg_nlevels = maxdepth + 1;
             }
             __syncthreads();

@@ -378,3 +378,33 @@ def test_sorted_frontier_rebuild(bcmod, oracle_mod, sort_frontier):
         with bcmod.BCGraph.from_graph(g, strategy="we", sort_frontier=sort_frontier) as bg:
             check_bc(bg, g, src, oracle_mod)
             check_source(bg, g, 5 if src is None else int(src[1]), oracle_mod)
+
+
+def test_trace_source_levels(bcmod, oracle_mod):
+    """N2 per-level trace: frontier sizes equal the oracle's level sizes exactly."""
+    for key in ("c1", "c3", "c4"):
+        g = graph(key)
+        s = int(gg.CONFIGS[key].sources(g)[3])
+        with bcmod.BCGraph.from_graph(g, strategy="we") as bg:
+            tr = bg.trace_source(s)
+        ref = oracle_mod.single_source(g, s)
+        assert tr["num_levels"] == ref["num_levels"]
+        assert np.array_equal(tr["level_sizes"], ref["level_sizes"])
+        assert np.all(tr["fwd_cycles"] > 0)
+        assert np.all(tr["bwd_cycles"][1:-1] > 0) and tr["bwd_cycles"][0] == 0
+
+
+@pytest.mark.parametrize("flags", [(1, 0), (0, 1), (1, 1)])
+def test_extrapolate_and_normalize(bcmod, oracle_mod, flags):
+    """N3 post-processing: n/k estimator scaling and the (n-1)(n-2) normalisation."""
+    extrapolate, normalize = flags
+    g = graph("c1")
+    src = gg.sample_sources(g, 100, seed=8)
+    ref = oracle_mod.bc(g, src, nthreads=8)
+    if extrapolate:
+        ref = ref * g.n / src.size
+    if normalize:
+        ref = ref / ((g.n - 1) * (g.n - 2))
+    with bcmod.BCGraph.from_graph(g, extrapolate=extrapolate, normalize=normalize) as bg:
+        got = bg.compute(src)
+    assert np.max(np.abs(got - ref) / np.maximum(np.abs(ref), 1e-300)) < 1e-9
