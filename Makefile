@@ -5,13 +5,22 @@ PKG := paper_conf_sc_mclaughlinb14_b200
 ARCH := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := -O3 -std=c++17 -lineinfo $(ARCH) -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
            -Iinclude -Xptxas -v
-SRCS := $(PKG)/csrc/bc_api.cu $(PKG)/csrc/bc_kernels.cuh include/bc.h
+CSRC := $(PKG)/csrc
+HDRS := $(CSRC)/bc_kernels.cuh include/bc.h
+# one translation unit per level store (compiled in parallel: make -j)
+UNITS := bc_api bc_inst_directed bc_inst_levels bc_inst_gcodes bc_inst_scodes
+OBJS := $(UNITS:%=build/%.o)
 
 all: $(PKG)/libbc.so $(PKG)/libgraphgen.so oracle/liboracle.so
 
-$(PKG)/libbc.so: $(SRCS)
-	$(NVCC) $(NVFLAGS) -shared -o $@ $(PKG)/csrc/bc_api.cu 2> $(PKG)/csrc/ptxas.log || (cat $(PKG)/csrc/ptxas.log; false)
-	@grep -E "registers|spill" $(PKG)/csrc/ptxas.log | sed 's/^ptxas info    : //' | sort -u | head -20
+build/%.o: $(CSRC)/%.cu $(HDRS)
+	@mkdir -p build
+	$(NVCC) $(NVFLAGS) -c -o $@ $< 2> build/$*.ptxas.log || (cat build/$*.ptxas.log; false)
+
+$(PKG)/libbc.so: $(OBJS)
+	$(NVCC) $(ARCH) -shared -o $@ $(OBJS)
+	@cat $(UNITS:%=build/%.ptxas.log) > $(CSRC)/ptxas.log
+	@grep -E "registers|spill" $(CSRC)/ptxas.log | sed 's/^ptxas info    : //' | sort -u | head -20
 
 $(PKG)/libgraphgen.so: $(PKG)/graphgen_native.c
 	gcc -O2 -std=c99 -fPIC -shared -pthread -o $@ $<
@@ -20,6 +29,6 @@ oracle/liboracle.so: oracle/brandes_oracle.c
 	gcc -O2 -std=c99 -fPIC -shared -pthread -o $@ $<
 
 clean:
-	rm -f $(PKG)/libbc.so $(PKG)/libgraphgen.so oracle/liboracle.so
+	rm -rf build $(PKG)/libbc.so $(PKG)/libgraphgen.so oracle/liboracle.so
 
 .PHONY: all clean

@@ -89,6 +89,10 @@ typedef struct bc_options {
                                 estimator of total BC ("trivially adjusted for approximation",
                                 P:315, refs [3],[9])                                            */
     int32_t normalize;       /* 1: divide by (n-1)(n-2), the normalisation of P:74             */
+    int32_t succ_bits;       /* 0 = auto (on with level_store 3), 1 = on, -1 = off: one
+                                bit per arc (per source in flight) marks DAG successors
+                                during the forward scan (Jia et al.'s O(m) boolean array,
+                                P:129); the backward then reads only successor arcs          */
 } bc_options;
 
 typedef struct bc_stats {

@@ -33,7 +33,7 @@ class bc_options(ctypes.Structure):
                 ("seq_max_deg", ctypes.c_int32), ("level_store", ctypes.c_int32),
                 ("warp_max_deg", ctypes.c_int32), ("l2_persist", ctypes.c_int32),
                 ("sort_frontier", ctypes.c_int32), ("extrapolate", ctypes.c_int32),
-                ("normalize", ctypes.c_int32)]
+                ("normalize", ctypes.c_int32), ("succ_bits", ctypes.c_int32)]
 
 
 class bc_stats(ctypes.Structure):

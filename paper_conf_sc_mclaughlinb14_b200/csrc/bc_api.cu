@@ -69,6 +69,8 @@ struct bc_graph {
     uint32_t *gcodes = nullptr, *gfb = nullptr;
     int sort_frontier = 0, sort_min = 0, nb_words = 0;  // sorted-frontier rebuild (configure())
     uint32_t *nbits = nullptr;
+    int succ_bits = 0, sb_words = 0;                    // successor bitmap over arcs
+    uint32_t *sbits = nullptr;
     int code_words = 0, fb_words = 0;
     int seq_max_deg = 32;
     int warp_max_deg = 4096;
@@ -126,6 +128,7 @@ extern "C" void bc_default_options(bc_options *o) {
     o->l2_persist = 0;
     o->sort_frontier = 0;
     o->extrapolate = 0;
+    o->succ_bits = 0;
     o->normalize = 0;
     o->level_store = 0;
 }
@@ -143,7 +146,9 @@ static void free_workspace(bc_graph *g) {
     cudaFree(g->gcodes);
     cudaFree(g->gfb);
     cudaFree(g->nbits);
+    cudaFree(g->sbits);
     g->nbits = nullptr;
+    g->sbits = nullptr;
     g->bigq = nullptr;
     g->gcodes = g->gfb = nullptr;
     g->d = nullptr;
@@ -157,23 +162,17 @@ static size_t slot_bytes(const bc_graph *g) {
     const size_t gc = g->lstore == 3 ? 4 * ((size_t)g->code_words + (size_t)g->fb_words) : 0;
     return g->stride_n * ((g->lstore == 1 ? sizeof(int) : 0) + 2 * sizeof(double) + sizeof(int)) +
            g->stride_e * (sizeof(int) + 1) + g->stride_big * sizeof(int) + gc +
-           (g->sort_frontier ? 4 * (size_t)g->nb_words : 0);
-}
-
-template <bool DIR, class LV, bool EPOK>
-static const void *kernel_for(int nt) {
-    return nt == 1024  ? (const void *)bc_kernel<DIR, LV, 1024, EPOK>
-           : nt == 512 ? (const void *)bc_kernel<DIR, LV, 512, EPOK>
-           : nt == 128 ? (const void *)bc_kernel<DIR, LV, 128, EPOK>
-                       : (const void *)bc_kernel<DIR, LV, 256, EPOK>;
+           (g->sort_frontier ? 4 * (size_t)g->nb_words : 0) +
+           (g->succ_bits ? 4 * (size_t)g->sb_words : 0);
 }
 
 template <bool EPOK>
 static const void *pick_kernel(const bc_graph *g, int nt) {
-    if (g->directed) return kernel_for<true, GlobalLevels, EPOK>(nt);
-    if (g->lstore == 2) return kernel_for<false, SmemCodes, EPOK>(nt);
-    if (g->lstore == 3) return kernel_for<false, GlobalCodes, EPOK>(nt);
-    return kernel_for<false, GlobalLevels, EPOK>(nt);
+    const bool sb = g->succ_bits != 0;
+    if (g->directed) return kernel_directed(nt, EPOK, sb);
+    if (g->lstore == 2) return kernel_scodes(nt, EPOK, sb);
+    if (g->lstore == 3) return kernel_gcodes(nt, EPOK, sb);
+    return kernel_levels(nt, EPOK, sb);
 }
 
 // Choose level store, block size and shared memory for both launch kinds
@@ -207,6 +206,12 @@ static int configure(bc_graph *g) {
     g->sort_frontier = o.sort_frontier > 0 ? 1 : (o.sort_frontier < 0 ? 0 : (g->n >= (1 << 17)));
     if (g->lstore == 3) g->sort_frontier = 1;  // codes in HBM/L2 discover through the bitmap
     g->nb_words = (int)((((size_t)g->n + 31) / 32 + 31) & ~(size_t)31);
+    // the bitmap replaces a probe of the level store per backward arc by one bit read,
+    // at the price of an atomic OR per row in the forward pass: measured +6% on c5k
+    // (codes in HBM/L2), neutral on c5ws, -10..-16% against shared-memory codes
+    // (c2/c3/c4), so auto enables it only with level store 3
+    g->succ_bits = o.succ_bits > 0 || (o.succ_bits == 0 && g->lstore == 3);
+    g->sb_words = (int)((((size_t)g->nnz + 31) / 32 + 2 + 3) & ~(size_t)3);
     g->sort_min = std::max(1024, g->n / 64);
     g->code_words = g->lstore >= 2 ? (int)(code_bytes / 4) : 0;
     g->fb_words = g->lstore >= 2 ? (int)(fb_bytes / 4) : 0;
@@ -274,6 +279,10 @@ static int alloc_workspace(bc_graph *g) {
     CK(cudaMalloc(&g->ends, ns * g->stride_e * sizeof(int)));
     CK(cudaMalloc(&g->modes, ns * g->stride_e));
     CK(cudaMalloc(&g->bigq, ns * g->stride_big * sizeof(int)));
+    if (g->succ_bits) {
+        CK(cudaMalloc(&g->sbits, ns * (size_t)g->sb_words * 4));
+        CK(cudaMemset(g->sbits, 0, ns * (size_t)g->sb_words * 4));
+    }
     if (g->sort_frontier) {
         CK(cudaMalloc(&g->nbits, ns * (size_t)g->nb_words * 4));
         CK(cudaMemset(g->nbits, 0, ns * (size_t)g->nb_words * 4));
@@ -474,7 +483,7 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     const int old_slots = g->slots;
     const int realloc = o->inflight != old.inflight || o->level_store != old.level_store ||
                         o->block_threads != old.block_threads || o->warp_max_deg != old.warp_max_deg ||
-                        o->sort_frontier != old.sort_frontier;
+                        o->sort_frontier != old.sort_frontier || o->succ_bits != old.succ_bits;
     if (realloc) {
         rc = alloc_workspace(g);
         if (rc) return rc;
@@ -524,6 +533,9 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     p.stride_nb = (size_t)g->nb_words;
     p.nb_words = g->nb_words;
     p.sort_min = g->sort_min;
+    p.sbits = g->succ_bits ? g->sbits : nullptr;
+    p.stride_sb = (size_t)g->sb_words;
+    p.sb_words = g->sb_words;
     p.seq_max_deg = g->seq_max_deg;
     p.warp_max_deg = g->warp_max_deg;
     p.stats = g->stats;

@@ -1,0 +1,9 @@
+// bc_inst_directed.cu -- instantiates bc_kernel for the GlobalLevels level store (directed graphs) in
+// all block sizes / EP / successor-bitmap variants (one translation unit per store so
+// the library compiles in parallel).  No code of its own: see bc_kernels.cuh.
+#define BC_INSTANCE_TU
+#include "bc_kernels.cuh"
+
+namespace bcdev {
+const void *kernel_directed(int nt, bool epok, bool sb) { return kernel_table<true, GlobalLevels>(nt, epok, sb); }
+}  // namespace bcdev

@@ -1,0 +1,9 @@
+// bc_inst_gcodes.cu -- instantiates bc_kernel for the GlobalCodes level store in
+// all block sizes / EP / successor-bitmap variants (one translation unit per store so
+// the library compiles in parallel).  No code of its own: see bc_kernels.cuh.
+#define BC_INSTANCE_TU
+#include "bc_kernels.cuh"
+
+namespace bcdev {
+const void *kernel_gcodes(int nt, bool epok, bool sb) { return kernel_table<false, GlobalCodes>(nt, epok, sb); }
+}  // namespace bcdev

@@ -86,6 +86,9 @@ struct KParams {
     size_t stride_nb;
     int nb_words;
     int sort_min;        // rebuild a level in vertex order when it has >= sort_min vertices
+    uint32_t *sbits;     // per-slot successor bitmap over arcs (ArcBits), NULL = off
+    size_t stride_sb;
+    int sb_words;        // multiple of 4
     int seq_max_deg;     // rows up to this degree: owner thread, CSR order
     int warp_max_deg;    // rows up to this degree: one warp; longer: whole CTA
     // strategy
@@ -290,32 +293,65 @@ __device__ __forceinline__ double warp_sum(double v) {
 #define BC_UNROLL 4
 #endif
 
-// Arcs a, a+stride, ... < e of one row: stride 1 for a row owned by one thread
-// (CSR order), stride = #cooperating threads for warp/CTA rows.  BC_UNROLL arcs
-// per step so that many col loads and gathers are in flight; padding slots add
-// +0.0, which leaves the CSR-order sum bit-identical.
+// Successor bitmap over the arcs of one source (one bit per CSR position): the
+// O(m) boolean array of Jia et al., kept for SUCCESSORS.  mode 1 (forward,
+// WE level L): bit a is set when col[a] is, or is about to become, a level-(L+1)
+// vertex -- known exactly while the row is scanned (an unvisited neighbour of a
+// level-L vertex can only be discovered at L+1).  mode 2 (backward level L): only
+// arcs whose bit is set are visited, without a probe, and col is read only for
+// them.  mode 0: not used (EP levels, option off).
+struct ArcBits {
+    uint32_t *sb = nullptr;
+    int mode = 0;
+    int knext = 0;  // code of level L+1
+    int unv = 0;    // code of "unvisited"
+};
+
+// Arcs t, t+stride, ... of row [b, e) for `stride` cooperating threads (a warp or the
+// CTA).  The loop trip count is uniform over the cooperating threads (ballots).
+// Forward: col loads of step i+1 are issued before the gathers of step i are
+// consumed; padding slots probe vertex 0 and add +0.0.
 template <int U, class Probe, class Gather, class Claim, class Visit>
-__device__ __forceinline__ double strided_sum(const int *__restrict__ cols, int a, int e, int stride,
-                                              Probe &probe, Gather &gather, Claim &claim, Visit &visit) {
+__device__ __forceinline__ double coop_sum(const int *__restrict__ cols, int b, int e, int t, int stride,
+                                           const ArcBits &ab, Probe &probe, Gather &gather,
+                                           Claim &claim, Visit &visit) {
     double acc = 0.0;
-    // software pipeline: the col loads of step i+1 are issued before the gathers of
-    // step i are consumed (padding slots probe vertex 0 and add +0.0)
+    const int lane = threadIdx.x & 31;
+    if (ab.mode == 2) {
+        for (int base = b; base < e; base += U * stride) {
+            int u[U];
+            bool ok[U];
+            double g[U];
+#pragma unroll
+            for (int j = 0; j < U; ++j) {
+                const int a = base + t + j * stride;
+                ok[j] = a < e && ((__ldcg(&ab.sb[a >> 5]) >> (a & 31)) & 1u);
+            }
+#pragma unroll
+            for (int j = 0; j < U; ++j) u[j] = ok[j] ? cols[base + t + j * stride] : 0;
+#pragma unroll
+            for (int j = 0; j < U; ++j) g[j] = ok[j] ? gather(u[j], ab.knext) : 0.0;
+#pragma unroll
+            for (int j = 0; j < U; ++j) acc += g[j];
+        }
+        return acc;
+    }
     int un[U];
 #pragma unroll
-    for (int j = 0; j < U; ++j) un[j] = a + j * stride < e ? cols[a + j * stride] : 0;
-    for (; a < e; a += U * stride) {
+    for (int j = 0; j < U; ++j) un[j] = b + t + j * stride < e ? cols[b + t + j * stride] : 0;
+    for (int base = b; base < e; base += U * stride) {
         int u[U], k[U];
         bool ok[U];
         double g[U];
 #pragma unroll
         for (int j = 0; j < U; ++j) {
             u[j] = un[j];
-            ok[j] = a + j * stride < e;
+            ok[j] = base + t + j * stride < e;
         }
-        const int an = a + U * stride;
-        if (an < e) {
+        const int bn = base + U * stride;
+        if (bn < e) {
 #pragma unroll
-            for (int j = 0; j < U; ++j) un[j] = an + j * stride < e ? cols[an + j * stride] : 0;
+            for (int j = 0; j < U; ++j) un[j] = bn + t + j * stride < e ? cols[bn + t + j * stride] : 0;
         }
 #pragma unroll
         for (int j = 0; j < U; ++j) k[j] = probe(u[j]);
@@ -327,6 +363,18 @@ __device__ __forceinline__ double strided_sum(const int *__restrict__ cols, int 
 #pragma unroll
         for (int j = 0; j < U; ++j)
             if (ok[j]) visit(u[j], k[j], won[j]);
+        if (ab.mode == 1) {
+#pragma unroll
+            for (int j = 0; j < U; ++j) {
+                const unsigned m = __ballot_sync(FULL, ok[j] && (k[j] == ab.unv || k[j] == ab.knext));
+                if (lane == 0 && m) {  // the warp's 32 arcs are consecutive
+                    const int A = base + j * stride + (t - lane);
+                    const int sh = A & 31;
+                    atomicOr(&ab.sb[A >> 5], m << sh);
+                    if (sh) atomicOr(&ab.sb[(A >> 5) + 1], m >> (32 - sh));
+                }
+            }
+        }
 #pragma unroll
         for (int j = 0; j < U; ++j) acc += g[j];
     }
@@ -335,20 +383,59 @@ __device__ __forceinline__ double strided_sum(const int *__restrict__ cols, int 
 
 // One row owned by one thread, read as aligned 16-byte quads of col (one LDG.128
 // per 4 arcs instead of four LDG.32 that each touch a different sector per lane).
-// Slots outside [a, e) probe vertex 0 and add +0.0, so the sum keeps the CSR order.
+// Slots outside [a, e) probe vertex 0 and add +0.0, so the sum keeps the CSR order
+// (also in mode 2, which skips non-successor slots: they only ever added 0.0).
 // cols must be 16-byte aligned with >= 3 ints of readable slack after the end.
 template <class Probe, class Gather, class Claim, class Visit>
-__device__ __forceinline__ double seq_row(const int *__restrict__ cols, int a, int e, Probe &probe,
-                                          Gather &gather, Claim &claim, Visit &visit) {
+__device__ __forceinline__ double seq_row(const int *__restrict__ cols, int a, int e, const ArcBits &ab,
+                                          Probe &probe, Gather &gather, Claim &claim, Visit &visit) {
     double acc = 0.0;
+    // Successor bits of the row through a 64-arc window of two bitmap words starting at
+    // word w0: loaded once (mode 2) / OR-ed once (mode 1) per row of <= 32 arcs.
+    int w0 = a >> 5;
+    uint64_t win = 0;
+    if (ab.mode == 2) {
+        win = __ldcg(&ab.sb[w0]);
+        if (e > (w0 + 1) * 32) win |= (uint64_t)__ldcg(&ab.sb[w0 + 1]) << 32;
+    }
     for (int q = a & ~3; q < e; q += 4) {
+        // in-row slots of this quad as a 4-bit mask
+        unsigned valid = 0xFu;
+        if (q < a) valid &= 0xFu << (a - q);
+        if (q + 4 > e) valid &= 0xFu >> (q + 4 - e);
+        int off = q - w0 * 32;
+        if (off >= 64) {  // rows longer than the window (seq_max_deg > 32)
+            if (ab.mode == 1) {
+                if ((uint32_t)win) atomicOr(&ab.sb[w0], (uint32_t)win);
+                if (win >> 32) atomicOr(&ab.sb[w0 + 1], (uint32_t)(win >> 32));
+            }
+            w0 += 2;
+            off -= 64;
+            win = 0;
+            if (ab.mode == 2) {
+                win = __ldcg(&ab.sb[w0]);
+                if (e > (w0 + 1) * 32) win |= (uint64_t)__ldcg(&ab.sb[w0 + 1]) << 32;
+            }
+        }
+        if (ab.mode == 2) {
+            const unsigned bits = (unsigned)(win >> off) & valid;
+            if (!bits) continue;
+            const int4 c4 = *reinterpret_cast<const int4 *>(cols + q);
+            const int u[4] = {c4.x, c4.y, c4.z, c4.w};
+            double g[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) g[j] = (bits >> j) & 1u ? gather(u[j], ab.knext) : 0.0;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) acc += g[j];
+            continue;
+        }
         const int4 c4 = *reinterpret_cast<const int4 *>(cols + q);
         int u[4] = {c4.x, c4.y, c4.z, c4.w}, k[4];
         bool ok[4];
         double g[4];
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
-            ok[j] = q + j >= a && q + j < e;
+            ok[j] = (valid >> j) & 1u;
             u[j] = ok[j] ? u[j] : 0;
         }
 #pragma unroll
@@ -361,8 +448,18 @@ __device__ __forceinline__ double seq_row(const int *__restrict__ cols, int a, i
 #pragma unroll
         for (int j = 0; j < 4; ++j)
             if (ok[j]) visit(u[j], k[j], won[j]);
+        if (ab.mode == 1) {
+            unsigned bits = 0;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) bits |= (ok[j] && (k[j] == ab.unv || k[j] == ab.knext)) ? 1u << j : 0u;
+            win |= (uint64_t)bits << off;
+        }
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc += g[j];
+    }
+    if (ab.mode == 1) {
+        if ((uint32_t)win) atomicOr(&ab.sb[w0], (uint32_t)win);
+        if (win >> 32) atomicOr(&ab.sb[w0 + 1], (uint32_t)(win >> 32));
     }
     return acc;
 }
@@ -380,8 +477,8 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
                                          const int *__restrict__ rows,
                                          const int *__restrict__ cols, int seq_max, int warp_max,
                                          int *__restrict__ bigq, Smem<NT> &sm, Counters &c,
-                                         Probe probe, Gather gather, Claim claim, Visit visit, Pre pre,
-                                         Finish finish) {
+                                         const ArcBits &ab, Probe probe, Gather gather, Claim claim,
+                                         Visit visit, Pre pre, Finish finish) {
     constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     // Phase A: each warp walks its own 32-vertex chunks; no CTA barrier.
@@ -397,7 +494,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
         // (1) short rows: owner thread, CSR order; gathers issued before side effects
         if (v >= 0 && deg <= seq_max) {
             const double pv = pre(v);
-            const double acc = seq_row(cols, beg, beg + deg, probe, gather, claim, visit);
+            const double acc = seq_row(cols, beg, beg + deg, ab, probe, gather, claim, visit);
             finish(v, acc, false, pv);
         }
         // (2) medium rows: the lanes of this warp take their rows one at a time
@@ -409,7 +506,8 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             const int b = __shfl_sync(FULL, beg, leader);
             const int e = b + __shfl_sync(FULL, deg, leader);
             const double pv = pre(w);
-            const double acc = warp_sum(strided_sum<BC_UNROLL>(cols, b + lane, e, 32, probe, gather, claim, visit));
+            const double acc =
+                warp_sum(coop_sum<BC_UNROLL>(cols, b, e, lane, 32, ab, probe, gather, claim, visit));
             if (lane == leader) finish(w, acc, true, pv);
         }
         // (3) long rows: queued for the CTA-cooperative phase B
@@ -423,7 +521,7 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
             const int b = rows[v], e = rows[v + 1];
             const double pv = pre(v);
             const double acc =
-                warp_sum(strided_sum<BC_UNROLL>(cols, b + threadIdx.x, e, NT, probe, gather, claim, visit));
+                warp_sum(coop_sum<BC_UNROLL>(cols, b, e, threadIdx.x, NT, ab, probe, gather, claim, visit));
             if (lane == 0) sm.red[wid] = acc;
             __syncthreads();
             if (threadIdx.x == 0) {
@@ -503,9 +601,16 @@ __device__ __forceinline__ int compact_level(uint32_t *nb, int words, int *out, 
 
 template <bool DIR, int NT, class LV>
 __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S, int *bigq,
-                           uint32_t *nb, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
+                           uint32_t *nb, uint32_t *sb, int L, int lo, int hi, Smem<NT> &sm,
+                           Counters &c) {
     const int L1 = L + 1;
     const int kprev = LV::key(L - 1);
+    ArcBits ab;  // successor bits written during the discovery scan (mode 1)
+    ab.sb = sb;
+    ab.mode = sb ? 1 : 0;
+    ab.knext = LV::key(L1);
+    ab.unv = LV::UNVISITED;
+    const ArcBits none_ab;
     auto probe = [&](int u) -> int { return lv.probe(u); };
     auto pull = [&](int u, int k) -> double { return k == kprev ? __ldcg(&sigma[u]) : 0.0; };
     auto claim = [&](int u, int k) -> bool {
@@ -542,22 +647,22 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
             if (L > 0) fin(v, acc, coop, 0.0);
         };
         const unsigned before = c.scanned;
-        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, pull,
-                     claim, visit, nopre, fin0);
+        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, ab, probe,
+                     pull, claim, visit, nopre, fin0);
         c.arcs_reached += c.scanned - before;
     } else {
         auto none = [&](int, int) -> double { return 0.0; };
         auto fin1 = [&](int, double, bool, double) {};
         const unsigned before = c.scanned;
-        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, none,
-                     claim, discover, nopre, fin1);
+        row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, ab, probe,
+                     none, claim, discover, nopre, fin1);
         c.arcs_reached += c.scanned - before;
         if (L > 0) {
             auto count = [&](int, int k, bool) {
                 if (k == kprev) c.dag++;
             };
-            row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe,
-                         pull, noclaim, count, nopre, fin);
+            row_pass<NT>(S, lo, hi, p.iro, p.icol, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, none_ab,
+                         probe, pull, noclaim, count, nopre, fin);
         }
     }
 }
@@ -656,15 +761,20 @@ __device__ __forceinline__ void finish_dependency(const KParams &p, double sw, d
 
 template <int NT, class LV>
 __device__ void backward_we(const KParams &p, const LV &lv, double *sig_om, const int *S, int *bigq,
-                            int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
+                            uint32_t *sb, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int knext = LV::key(L + 1);
+    ArcBits ab;  // successors from the forward's bits (mode 2): no probe, col only for them
+    ab.sb = sb;
+    ab.mode = sb ? 2 : 0;
+    ab.knext = knext;
+    ab.unv = LV::UNVISITED;
     auto probe = [&](int v) -> int { return lv.probe(v); };
     auto gather = [&](int v, int k) -> double { return k == knext ? __ldcg(&sig_om[v]) : 0.0; };
     auto noclaim = [&](int, int) -> bool { return false; };
     auto none = [&](int, int, bool) {};
     auto pre = [&](int w) -> double { return __ldcg(&sig_om[w]); };  // sigma[w], issued early
     auto fin = [&](int w, double acc, bool, double sw) { finish_dependency(p, sw, sig_om, w, acc); };
-    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, probe, gather,
+    row_pass<NT>(S, lo, hi, p.ro, p.col, p.seq_max_deg, p.warp_max_deg, bigq, sm, c, ab, probe, gather,
                  noclaim, none, pre, fin);
 }
 
@@ -714,8 +824,9 @@ template <> __device__ __forceinline__ GlobalCodes make_levels<GlobalCodes>(cons
 }
 
 // EPOK = false instantiates a work-efficient-only kernel (no EP code, fewer
-// registers) for launches that never run an EP level.
-template <bool DIR, class LV, int NT, bool EPOK>
+// registers) for launches that never run an EP level.  SB = false compiles the
+// successor bitmap out (it costs registers even when p.sbits is NULL).
+template <bool DIR, class LV, int NT, bool EPOK, bool SB>
 #ifndef BC_MINB512
 #define BC_MINB512 2
 #endif
@@ -732,6 +843,7 @@ bc_kernel(KParams p) {
     unsigned char *modes = p.modes + slot * p.stride_e;
     int *bigq = p.bigq + slot * p.stride_big;
     uint32_t *nb = p.nbits ? p.nbits + slot * p.stride_nb : nullptr;
+    uint32_t *sb = SB && p.sbits ? p.sbits + slot * p.stride_sb : nullptr;
 
     Counters c;
     const int run_ep = (p.launch_mode == LM_SAMPLED && p.sampled_flag) ? *p.sampled_flag : 0;
@@ -770,7 +882,7 @@ bc_kernel(KParams p) {
             uint32_t *const nbl =
                 LV::BITMAP_DISCOVERY ? nb
                                      : ((nb && (long long)(hi - lo) * 4 >= p.sort_min) ? nb : nullptr);
-            if (!EPOK || mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, nbl, L, lo, hi, sm, c);
+            if (!EPOK || mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, nbl, sb, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             // (the level functions end with a barrier: every discovery is recorded)
             int nhi;
@@ -830,7 +942,9 @@ bc_kernel(KParams p) {
             const int blo = ends[Lb], bhi = ends[Lb + 1];
             const int bmode = p.backward_we ? MODE_WE : (int)modes[Lb];
             const long long t0 = clock64();
-            if (!EPOK || bmode == MODE_WE) backward_we<NT>(p, lv, sigma, S, bigq, Lb, blo, bhi, sm, c);
+            // the forward's successor bits exist only if forward level Lb ran WE
+            uint32_t *const sbl = (sb && (!EPOK || modes[Lb] == MODE_WE)) ? sb : nullptr;
+            if (!EPOK || bmode == MODE_WE) backward_we<NT>(p, lv, sigma, S, bigq, sbl, Lb, blo, bhi, sm, c);
             else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
             if (threadIdx.x == 0) {
                 const long long dt = clock64() - t0;
@@ -856,6 +970,10 @@ bc_kernel(KParams p) {
         if (LV::RESET_VERTICES)
             for (int i = threadIdx.x; i < S_len; i += NT) lv.reset_vertex(S[i]);
         lv.template reset_all<NT>(p.code_words);
+        if (sb) {  // successor bits of this source
+            uint4 *s4 = reinterpret_cast<uint4 *>(sb);
+            for (int i = threadIdx.x; i < (p.sb_words >> 2); i += NT) s4[i] = make_uint4(0u, 0u, 0u, 0u);
+        }
         flush_counters(c, sm.st);
         if (threadIdx.x == 0) {
             sm.st.src += 1;
@@ -880,6 +998,29 @@ bc_kernel(KParams p) {
     }
 }
 
+// Address of bc_kernel<DIR, LV, nt, epok, sb> (host side).  Each level store is
+// instantiated in its own translation unit (bc_inst_*.cu) so the library builds in
+// parallel; bc_api.cu reaches them through the kernel_* functions declared below.
+template <bool DIR, class LV, int NT>
+const void *kernel_nt(bool epok, bool sb) {
+    return epok ? (sb ? (const void *)bc_kernel<DIR, LV, NT, true, true>
+                      : (const void *)bc_kernel<DIR, LV, NT, true, false>)
+                : (sb ? (const void *)bc_kernel<DIR, LV, NT, false, true>
+                      : (const void *)bc_kernel<DIR, LV, NT, false, false>);
+}
+template <bool DIR, class LV>
+const void *kernel_table(int nt, bool epok, bool sb) {
+    return nt == 1024  ? kernel_nt<DIR, LV, 1024>(epok, sb)
+           : nt == 512 ? kernel_nt<DIR, LV, 512>(epok, sb)
+           : nt == 128 ? kernel_nt<DIR, LV, 128>(epok, sb)
+                       : kernel_nt<DIR, LV, 256>(epok, sb);
+}
+const void *kernel_directed(int nt, bool epok, bool sb);       // GlobalLevels, DIR
+const void *kernel_levels(int nt, bool epok, bool sb);         // GlobalLevels, undirected
+const void *kernel_gcodes(int nt, bool epok, bool sb);         // GlobalCodes
+const void *kernel_scodes(int nt, bool epok, bool sb);         // SmemCodes
+
+#ifndef BC_INSTANCE_TU
 // Alg. 5 decision: sort keys ascending, median = keys[nk/2],
 // EP iff median < gamma*log2(n).  One CTA, bitonic sort in shared memory.
 __global__ void __launch_bounds__(1024) sampling_decide_kernel(const int *keys, int nk,
@@ -937,5 +1078,7 @@ __global__ void unpermute_kernel(const double *__restrict__ bc_int, const int *_
          i += (long long)gridDim.x * blockDim.x)
         out[i] = f * bc_int[perm[i]];
 }
+
+#endif  // BC_INSTANCE_TU
 
 }  // namespace bcdev

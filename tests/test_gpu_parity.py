@@ -380,6 +380,23 @@ def test_sorted_frontier_rebuild(bcmod, oracle_mod, sort_frontier):
             check_source(bg, g, 5 if src is None else int(src[1]), oracle_mod)
 
 
+@pytest.mark.parametrize("succ_bits", [-1, 1])
+@pytest.mark.parametrize("case", [("c1", "we", 0), ("c1", "hybrid", 0), ("c2d", "we", 0),
+                                  ("c3", "we", 3), ("c4", "we", 2), ("c4", "we", 3),
+                                  ("c4", "ep", 0), ("c4", "sampling", 1)])
+def test_successor_bitmap(bcmod, oracle_mod, succ_bits, case):
+    """The successor bitmap (one bit per arc set in the forward scan, read by the backward
+    sweep) only skips non-successor arcs: d/sigma/delta and BC are unchanged."""
+    key, strategy, lstore = case
+    g = graph(key)
+    src = gg.CONFIGS[key].sources(g)[:150]
+    with bcmod.BCGraph.from_graph(g, strategy=strategy, succ_bits=succ_bits,
+                                  level_store=lstore) as bg:
+        check_bc(bg, g, src, oracle_mod)
+        check_source(bg, g, int(src[2]), oracle_mod)
+        check_source(bg, g, int(src[2]), oracle_mod)  # bitmap cleared between sources
+
+
 def test_trace_source_levels(bcmod, oracle_mod):
     """N2 per-level trace: frontier sizes equal the oracle's level sizes exactly."""
     for key in ("c1", "c3", "c4"):
