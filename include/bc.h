@@ -59,6 +59,19 @@ enum {
     BC_STRATEGY_SAMPLING = 3  /* Alg. 5: median max-depth of n_samps WE roots < gamma*log2(n) */
 };
 
+/* Execution engine (how sources are scheduled; results are the same up to fp64 rounding). */
+enum {
+    BC_ENGINE_AUTO = 0,       /* per-source engine, except that a SAMPLING run whose Alg. 5
+                                 decision is EP ("small-world": median depth < gamma*log2 n)
+                                 on an undirected graph runs its main phase batched          */
+    BC_ENGINE_PER_SOURCE = 1, /* one CTA per source (bc_kernel), every level WE or EP as the
+                                 strategy chooses                                            */
+    BC_ENGINE_BATCHED = 2     /* undirected graphs: 64 sources per batch, level-synchronous
+                                 over the whole GPU, one 64-bit source mask per vertex and
+                                 level; every union-frontier row is read once per level for
+                                 all 64 sources (work-efficient, queue-driven expansion)    */
+};
+
 typedef struct bc_graph bc_graph; /* opaque; owns device copies of the graph and workspace */
 
 typedef struct bc_options {
@@ -93,6 +106,11 @@ typedef struct bc_options {
                                 bit per arc (per source in flight) marks DAG successors
                                 during the forward scan (Jia et al.'s O(m) boolean array,
                                 P:129); the backward then reads only successor arcs          */
+    int32_t engine;          /* BC_ENGINE_*, default BC_ENGINE_AUTO                            */
+    int32_t batch_levels;    /* batched engine: BFS levels a batch may have (0 = auto 64, max
+                                254); sources of a deeper batch are rerun per source         */
+    int32_t hub_chunk;       /* batched engine: rows longer than this are split into chunks of
+                                this many arcs spread over the GPU (0 = auto 1024)            */
 } bc_options;
 
 typedef struct bc_stats {
@@ -113,6 +131,8 @@ typedef struct bc_stats {
     double kernel_ms;         /* summed CUDA-event time of the bc_kernel launches             */
     int64_t phase_cycles[4];  /* SM cycles summed over CTAs in forward WE, forward EP,
                                  backward WE, backward EP levels (device trace)               */
+    int64_t batches;          /* batches of 64 sources run by the batched engine (0: not run) */
+    int64_t batch_overflows;  /* ... of which exceeded batch_levels and were rerun per source */
 } bc_stats;
 
 /* Copy a CSR graph to `device` and allocate the per-source workspace.
@@ -164,6 +184,17 @@ BC_API int bc_single_source(bc_graph *g, int32_t s, int32_t *d, double *sigma, d
  *   num_levels   receives maxdepth + 1 (arrays hold min(max_levels, num_levels) entries) */
 BC_API int bc_trace_source(bc_graph *g, int32_t s, int32_t *level_sizes, int64_t *fwd_cycles,
                            int64_t *bwd_cycles, int32_t max_levels, int32_t *num_levels);
+
+/* Debug/parity export of the batched engine for one batch of 1..64 sources (undirected
+ * graphs): runs exactly the kernel bc_compute uses in batched mode, with per-source
+ * outputs.  Host arrays, row b = sources[b], each may be NULL:
+ *   d      int32[k][n]   BFS distance from sources[b], -1 = unreachable
+ *   sigma  double[k][n]  shortest-path counts (0 if unreachable)
+ *   delta  double[k][n]  dependencies (0 for the source, unreachable and deepest vertices)
+ * BC_EINVAL for a directed graph, k outside 1..64, an out-of-range source, or a batch
+ * deeper than batch_levels. */
+BC_API int bc_batch_sources(bc_graph *g, const int32_t *sources, int32_t k, int32_t *d,
+                            double *sigma, double *delta);
 
 BC_API void bc_default_options(bc_options *o);
 BC_API int bc_set_options(bc_graph *g, const bc_options *o); /* validates; may reallocate workspace */

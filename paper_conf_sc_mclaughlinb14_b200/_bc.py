@@ -19,9 +19,12 @@ LIB_PATH = os.path.join(_HERE, "libbc.so")
 BC_OK, BC_EINVAL, BC_ENOMEM, BC_ECUDA, BC_EINTERNAL = 0, -1, -2, -3, -4
 BC_STRATEGY_WE, BC_STRATEGY_EP, BC_STRATEGY_HYBRID, BC_STRATEGY_SAMPLING = 0, 1, 2, 3
 STRATEGIES = {"we": 0, "ep": 1, "hybrid": 2, "sampling": 3}
+BC_ENGINE_AUTO, BC_ENGINE_PER_SOURCE, BC_ENGINE_BATCHED = 0, 1, 2
+ENGINES = {"auto": 0, "per_source": 1, "batched": 2}
+BATCH_WIDTH = 64  # sources per batch of the batched engine
 
 EXPORTED = ("bc_graph_create", "bc_compute", "bc_compute_device", "bc_single_source",
-            "bc_trace_source", "bc_default_options", "bc_set_options", "bc_get_options",
+            "bc_trace_source", "bc_batch_sources", "bc_default_options", "bc_set_options", "bc_get_options",
             "bc_get_stats", "bc_destroy", "bc_last_error")
 
 
@@ -33,7 +36,9 @@ class bc_options(ctypes.Structure):
                 ("seq_max_deg", ctypes.c_int32), ("level_store", ctypes.c_int32),
                 ("warp_max_deg", ctypes.c_int32), ("l2_persist", ctypes.c_int32),
                 ("sort_frontier", ctypes.c_int32), ("extrapolate", ctypes.c_int32),
-                ("normalize", ctypes.c_int32), ("succ_bits", ctypes.c_int32)]
+                ("normalize", ctypes.c_int32), ("succ_bits", ctypes.c_int32),
+                ("engine", ctypes.c_int32), ("batch_levels", ctypes.c_int32),
+                ("hub_chunk", ctypes.c_int32)]
 
 
 class bc_stats(ctypes.Structure):
@@ -44,7 +49,8 @@ class bc_stats(ctypes.Structure):
                 ("sampling_ep", ctypes.c_int32), ("sampling_median", ctypes.c_int32),
                 ("sigma_inexact", ctypes.c_int32), ("inflight", ctypes.c_int32),
                 ("kernel_launches", ctypes.c_int32), ("bc_kernel_launches", ctypes.c_int32),
-                ("kernel_ms", ctypes.c_double), ("phase_cycles", ctypes.c_int64 * 4)]
+                ("kernel_ms", ctypes.c_double), ("phase_cycles", ctypes.c_int64 * 4),
+                ("batches", ctypes.c_int64), ("batch_overflows", ctypes.c_int64)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_}
@@ -82,6 +88,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.bc_single_source.argtypes = [_vp, ctypes.c_int32, _i32p, _f64p, _f64p, _u8p,
                                      ctypes.c_int32, _i32p]
     lib.bc_trace_source.argtypes = [_vp, ctypes.c_int32, _i32p, _i64p, _i64p, ctypes.c_int32, _i32p]
+    lib.bc_batch_sources.argtypes = [_vp, _i32p, ctypes.c_int32, _i32p, _f64p, _f64p]
     lib.bc_default_options.argtypes = [ctypes.POINTER(bc_options)]
     lib.bc_default_options.restype = None
     lib.bc_set_options.argtypes = [_vp, ctypes.POINTER(bc_options)]
@@ -92,7 +99,8 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.bc_last_error.argtypes = []
     lib.bc_last_error.restype = ctypes.c_char_p
     for name in ("bc_graph_create", "bc_compute", "bc_compute_device", "bc_single_source",
-                 "bc_trace_source", "bc_set_options", "bc_get_options", "bc_get_stats"):
+                 "bc_trace_source", "bc_batch_sources", "bc_set_options", "bc_get_options",
+                 "bc_get_stats"):
         getattr(lib, name).restype = ctypes.c_int
     _lib = lib
     return lib
@@ -173,6 +181,19 @@ def bc_trace_source(handle: int, s: int, max_levels: int = 1 << 16) -> dict:
                 num_levels=nl.value)
 
 
+def bc_batch_sources(handle: int, n: int, sources) -> dict:
+    """Per-source d / sigma / delta of one batch (1..64 sources) of the batched engine."""
+    lib = load_library()
+    src = np.ascontiguousarray(sources, dtype=np.int32)
+    k = int(src.size)
+    d = np.empty((k, n), dtype=np.int32)
+    sigma = np.empty((k, n), dtype=np.float64)
+    delta = np.empty((k, n), dtype=np.float64)
+    _check(lib.bc_batch_sources(_vp(handle), _ptr(src, _i32p), k, _ptr(d, _i32p), _ptr(sigma, _f64p),
+                                _ptr(delta, _f64p)))
+    return dict(d=d, sigma=sigma, delta=delta)
+
+
 def bc_default_options() -> bc_options:
     o = bc_options()
     load_library().bc_default_options(ctypes.byref(o))
@@ -224,6 +245,8 @@ class BCGraph:
         for k, v in kw.items():
             if k == "strategy" and isinstance(v, str):
                 v = STRATEGIES[v]
+            if k == "engine" and isinstance(v, str):
+                v = ENGINES[v]
             if not hasattr(o, k):
                 raise KeyError(k)
             setattr(o, k, v)
@@ -247,6 +270,9 @@ class BCGraph:
 
     def single_source(self, s: int, max_levels: Optional[int] = None) -> dict:
         return bc_single_source(self.handle, self.n, s, max_levels)
+
+    def batch_sources(self, sources) -> dict:
+        return bc_batch_sources(self.handle, self.n, sources)
 
     def trace_source(self, s: int, max_levels: int = 1 << 16) -> dict:
         return bc_trace_source(self.handle, s, max_levels)

@@ -6,6 +6,7 @@
 // kernels of bc_kernels.cuh; this file only validates, copies and launches.
 #include "bc.h"
 #include "bc_kernels.cuh"
+#include "bc_batch.cuh"
 
 #include <algorithm>
 #include <cmath>
@@ -110,6 +111,20 @@ struct bc_graph {
     int bc_launches = 0;     // ... of which bc_kernel
     cudaEvent_t tev[4] = {nullptr, nullptr, nullptr, nullptr};  // around the bc_kernel launches
     int tev_used[2] = {0, 0};
+    // multi-source batched engine (bc_batch.cu); allocated on first use
+    std::vector<int> h_ro;              // internal CSR offsets (hub counts for any chunk size)
+    struct Batch {
+        int ready = 0, failed = 0;
+        int Lcap = 0, LS = 0, CH = 0, nt = 256, grid = 0;
+        long long qcap = 0, hcap = 0;
+        unsigned long long *F = nullptr, *hcnt = nullptr, *lvor = nullptr;
+        double *sig = nullptr, *hacc = nullptr;
+        int *Q = nullptr, *qcnt = nullptr, *grab = nullptr, *hv = nullptr, *hb = nullptr;
+        int *ovf_src = nullptr;
+        long long ovf_cap = 0;
+        long long *ovf_n = nullptr;
+    } bt;
+    int batch_ran = 0;       // the last compute call launched the batched engine
 };
 
 extern "C" void bc_default_options(bc_options *o) {
@@ -131,6 +146,9 @@ extern "C" void bc_default_options(bc_options *o) {
     o->succ_bits = 0;
     o->normalize = 0;
     o->level_store = 0;
+    o->engine = BC_ENGINE_AUTO;
+    o->batch_levels = 0;
+    o->hub_chunk = 0;
 }
 
 extern "C" const char *bc_last_error(void) { return g_err; }
@@ -294,11 +312,149 @@ static int alloc_workspace(bc_graph *g) {
     return BC_OK;
 }
 
+static void free_batch(bc_graph *g) {
+    bc_graph::Batch &b = g->bt;
+    cudaFree(b.F);
+    cudaFree(b.hcnt);
+    cudaFree(b.lvor);
+    cudaFree(b.sig);
+    cudaFree(b.hacc);
+    cudaFree(b.Q);
+    cudaFree(b.qcnt);
+    cudaFree(b.grab);
+    cudaFree(b.hv);
+    cudaFree(b.hb);
+    cudaFree(b.ovf_src);
+    cudaFree(b.ovf_n);
+    b = bc_graph::Batch{};
+}
+
+// Workspace of the batched engine: vertex-major level masks F[(Lcap + 2) n], sigma/omega
+// [n][64], the union-frontier lists Q (a vertex is in at most min(64, Lcap + 2) of them),
+// hub entries and their partial sums.  Sized on first use; ~1.3 KB per vertex at Lcap 64.
+static int alloc_batch(bc_graph *g, long long max_sources) {
+    bc_graph::Batch &b = g->bt;
+    const int Lcap = g->opt.batch_levels > 0 ? g->opt.batch_levels : 64;
+    const int CH = g->opt.hub_chunk > 0 ? g->opt.hub_chunk : 1024;
+    const long long ovf_need = std::max<long long>(max_sources, 64);
+    if (b.ready && b.Lcap == Lcap && b.CH == CH && b.ovf_cap >= ovf_need) return BC_OK;
+    free_batch(g);
+    const size_t n = (size_t)std::max(g->n, 1);
+    b.Lcap = Lcap;
+    b.LS = Lcap + 2;
+    b.CH = CH;
+    long long nhub = 0;
+    for (int v = 0; v < g->n; ++v) nhub += (g->h_ro[v + 1] - g->h_ro[v]) > CH;
+    const long long per_v = std::min(bcbatch::BW, b.LS);
+    b.qcap = (long long)n * per_v;
+    b.hcap = std::max<long long>(1, nhub * per_v);
+    b.ovf_cap = ovf_need;
+    CK(cudaMalloc(&b.F, n * (size_t)b.LS * 8));
+    CK(cudaMalloc(&b.sig, n * bcbatch::BW * sizeof(double)));
+    CK(cudaMalloc(&b.Q, (size_t)b.qcap * sizeof(int)));
+    CK(cudaMalloc(&b.qcnt, (size_t)b.LS * sizeof(int)));
+    CK(cudaMalloc(&b.hcnt, (size_t)b.LS * 8));
+    CK(cudaMalloc(&b.grab, 4 * (size_t)b.LS * sizeof(int)));
+    CK(cudaMalloc(&b.lvor, (size_t)b.LS * 8));
+    CK(cudaMalloc(&b.hv, (size_t)b.hcap * sizeof(int)));
+    CK(cudaMalloc(&b.hb, (size_t)b.hcap * sizeof(int)));
+    CK(cudaMalloc(&b.hacc, (size_t)b.hcap * bcbatch::BW * sizeof(double)));
+    CK(cudaMalloc(&b.ovf_src, (size_t)b.ovf_cap * sizeof(int)));
+    CK(cudaMalloc(&b.ovf_n, sizeof(long long)));
+    CK(cudaMemset(b.F, 0, n * (size_t)b.LS * 8));
+    CK(cudaMemset(b.qcnt, 0, (size_t)b.LS * sizeof(int)));
+    CK(cudaMemset(b.hcnt, 0, (size_t)b.LS * 8));
+    CK(cudaMemset(b.grab, 0, 4 * (size_t)b.LS * sizeof(int)));
+    CK(cudaMemset(b.lvor, 0, (size_t)b.LS * 8));
+    CK(cudaMemset(b.hacc, 0, (size_t)b.hcap * bcbatch::BW * sizeof(double)));
+    CK(cudaMemset(b.ovf_n, 0, sizeof(long long)));
+    b.nt = 256;
+    const void *fn = bcbatch::batch_kernel_fn(b.nt);
+    int per_sm = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, b.nt, 0));
+    if (per_sm < 1) return fail(BC_EINTERNAL, "batched kernel cannot be resident");
+    b.grid = per_sm * g->num_sms;
+    CK(cudaDeviceSynchronize());
+    b.ready = 1;
+    return BC_OK;
+}
+
+// Whether this call may run the batched engine (undirected graphs only: the
+// three-mask visited test relies on neighbours being on adjacent levels).
+static bool batch_wanted(const bc_graph *g) {
+    if (g->directed || g->n == 0) return false;
+    if (g->opt.engine == BC_ENGINE_BATCHED) return true;
+    return g->opt.engine == BC_ENGINE_AUTO && g->opt.strategy == BC_STRATEGY_SAMPLING;
+}
+
+static int launch_batch(bc_graph *g, const bcbatch::BParams &bp0, cudaStream_t st) {
+    if (bp0.k <= 0) return BC_OK;
+    bcbatch::BParams bp = bp0;
+    void *args[] = {&bp};
+    cudaLaunchConfig_t lc{};
+    lc.gridDim = dim3(g->bt.grid);
+    lc.blockDim = dim3(g->bt.nt);
+    lc.dynamicSmemBytes = 0;
+    lc.stream = st;
+    cudaLaunchAttribute attr[2];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    int na = 1;
+    if (g->l2win.num_bytes) {
+        attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[1].val.accessPolicyWindow = g->l2win;
+        na = 2;
+    }
+    lc.attrs = attr;
+    lc.numAttrs = na;
+    CK(cudaLaunchKernelExC(&lc, bcbatch::batch_kernel_fn(g->bt.nt), args));
+    g->launches++;
+    g->bc_launches++;
+    g->batch_ran = 1;
+    g->last_inflight = std::max(g->last_inflight, g->bt.grid);
+    return BC_OK;
+}
+
+static bcbatch::BParams batch_params(bc_graph *g, const int *d_sources, long long base, long long k,
+                                     double *acc_bc) {
+    const bc_graph::Batch &b = g->bt;
+    bcbatch::BParams bp;
+    memset(&bp, 0, sizeof(bp));
+    bp.n = g->n;
+    bp.ro = g->ro;
+    bp.col = g->col;
+    bp.sources = d_sources;
+    bp.perm = g->perm;
+    bp.src_base = base;
+    bp.k = k;
+    bp.Lcap = b.Lcap;
+    bp.LS = b.LS;
+    bp.CH = b.CH;
+    bp.F = b.F;
+    bp.sig = b.sig;
+    bp.Q = b.Q;
+    bp.qcap = b.qcap;
+    bp.qcnt = b.qcnt;
+    bp.hcnt = b.hcnt;
+    bp.grab = b.grab;
+    bp.lvor = b.lvor;
+    bp.hv = b.hv;
+    bp.hb = b.hb;
+    bp.hacc = b.hacc;
+    bp.hcap = b.hcap;
+    bp.bc = acc_bc;
+    bp.stats = g->stats;
+    bp.ovf_src = b.ovf_src;
+    bp.ovf_n = b.ovf_n;
+    return bp;
+}
+
 extern "C" void bc_destroy(bc_graph *g) {
     if (!g) return;
     DeviceGuard dg(g->device);
     if (g->done) cudaEventSynchronize(g->done);
     free_workspace(g);
+    free_batch(g);
     if (g->l2win.num_bytes) {
         cudaCtxResetPersistingL2Cache();
         cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
@@ -368,6 +524,7 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col_in) 
     } else {
         for (int v = 0; v <= n; ++v) ro32[v] = (int)ro64[v];
     }
+    g->h_ro = ro32;
     CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&g->done, cudaEventDisableTiming));
     for (auto &e : g->tev) CK(cudaEventCreate(&e));
@@ -405,7 +562,7 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col_in) 
             CK(cudaGetLastError());
         }
     }
-    CK(cudaMalloc(&g->counters, 2 * sizeof(unsigned long long)));
+    CK(cudaMalloc(&g->counters, 3 * sizeof(unsigned long long)));
     CK(cudaMalloc(&g->keys, sizeof(int) * 8192));
     CK(cudaMalloc(&g->flag, sizeof(int)));
     CK(cudaMemset(g->flag, 0, sizeof(int)));
@@ -465,7 +622,9 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     if (o->strategy < 0 || o->strategy > 3) return fail(BC_EINVAL, "bad strategy %d", o->strategy);
     if (o->n_samps < 1 || o->n_samps > 8192) return fail(BC_EINVAL, "n_samps must be in [1, 8192]");
     if (o->alpha < 0 || o->beta < 0 || o->ep_min_frontier < 0 || o->inflight < 0 || !(o->gamma >= 0) ||
-        o->seq_max_deg < 0 || o->warp_max_deg < 0 || o->level_store < 0 || o->level_store > 3)
+        o->seq_max_deg < 0 || o->warp_max_deg < 0 || o->level_store < 0 || o->level_store > 3 ||
+        o->engine < 0 || o->engine > 2 || o->batch_levels < 0 || o->batch_levels > bcbatch::MAX_LCAP ||
+        o->hub_chunk < 0)
         return fail(BC_EINVAL, "invalid parameter");
     if (o->block_threads != 0 && o->block_threads != 128 && o->block_threads != 256 &&
         o->block_threads != 512 && o->block_threads != 1024)
@@ -591,18 +750,22 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
     }
     double *acc_bc = g->perm ? g->bc_tmp : d_bc;  // accumulate in internal ids
     CK(cudaMemsetAsync(acc_bc, 0, sizeof(double) * (size_t)g->n, st));
-    CK(cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), st));
+    CK(cudaMemsetAsync(g->counters, 0, 3 * sizeof(unsigned long long), st));
     CK(cudaMemsetAsync(g->stats, 0, sizeof(DevStats), st));
     g->last_inflight = 0;
     g->launches = g->bc_launches = 0;
     g->tev_used[0] = g->tev_used[1] = 0;
+    g->batch_ran = 0;
     KParams p = base_params(g, acc_bc);
     p.sources = d_sources;
     int rc = BC_OK;
     const int strat = g->opt.strategy;
+    const int mode_main = strat == BC_STRATEGY_WE ? LM_WE : strat == BC_STRATEGY_EP ? LM_EP
+                        : strat == BC_STRATEGY_HYBRID ? LM_HYBRID : LM_SAMPLED;
+    long long ks = 0;
     if (strat == BC_STRATEGY_SAMPLING) {
         // Alg. 5: first n_samps sources WE, record max depth, decide, then the rest.
-        const long long ks = std::min<long long>(k, g->opt.n_samps);
+        ks = std::min<long long>(k, g->opt.n_samps);
         KParams ps = p;
         ps.launch_mode = LM_WE;
         ps.src_base = 0;
@@ -625,29 +788,51 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
             g->launches++;
             g->sampling_ran = 1;
         }
-        KParams pm = p;
-        pm.launch_mode = LM_SAMPLED;
-        pm.src_base = ks;
-        pm.k = k - ks;
-        pm.work_counter = g->counters + 1;
-        if (pm.k > 0) {
-            CK(cudaEventRecord(g->tev[2], st));
-            if ((rc = launch(g, pm, st))) return rc;
-            CK(cudaEventRecord(g->tev[3], st));
-            g->tev_used[1] = 1;
+    }
+    // Main phase.  With the batched engine in auto mode, both engines are enqueued and
+    // the device-side Alg. 5 decision picks one: an EP ("small-world") run goes to the
+    // multi-source batched kernel, a WE run to bc_kernel; sources of batches deeper than
+    // the level cap are rerun by bc_kernel (count read on the device).
+    const long long km = k - ks;
+    bool batched = km > 0 && batch_wanted(g);
+    if (batched && !g->bt.failed) {
+        rc = alloc_batch(g, km);
+        if (rc) {
+            if (g->opt.engine == BC_ENGINE_BATCHED) return rc;
+            g->bt.failed = 1;  // auto: keep the per-source engine
+            free_batch(g);
         }
-    } else {
-        KParams pm = p;
-        pm.launch_mode = strat == BC_STRATEGY_WE ? LM_WE : strat == BC_STRATEGY_EP ? LM_EP : LM_HYBRID;
-        pm.src_base = 0;
-        pm.k = k;
-        pm.work_counter = g->counters + 1;
-        if (pm.k > 0) {
-            CK(cudaEventRecord(g->tev[2], st));
+    }
+    batched = batched && g->bt.ready;
+    const bool gated = batched && g->opt.engine == BC_ENGINE_AUTO;  // decided by the Alg. 5 flag
+    if (km > 0) {
+        CK(cudaEventRecord(g->tev[2], st));
+        if (!batched || gated) {
+            KParams pm = p;
+            pm.launch_mode = mode_main;
+            pm.src_base = ks;
+            pm.k = km;
+            pm.work_counter = g->counters + 1;
+            pm.skip_if_ep = gated ? 1 : 0;
             if ((rc = launch(g, pm, st))) return rc;
-            CK(cudaEventRecord(g->tev[3], st));
-            g->tev_used[1] = 1;
         }
+        if (batched) {
+            CK(cudaMemsetAsync(g->bt.ovf_n, 0, sizeof(long long), st));
+            bcbatch::BParams bp = batch_params(g, d_sources, ks, km, acc_bc);
+            bp.sampled_flag = gated ? g->flag : nullptr;
+            if ((rc = launch_batch(g, bp, st))) return rc;
+            KParams po = p;  // overflow rerun (usually zero sources: the CTAs exit at once)
+            po.launch_mode = mode_main;
+            po.sources = g->bt.ovf_src;
+            po.perm = g->perm;
+            po.src_base = 0;
+            po.k = km;
+            po.k_dev = g->bt.ovf_n;
+            po.work_counter = g->counters + 2;
+            if ((rc = launch(g, po, st))) return rc;
+        }
+        CK(cudaEventRecord(g->tev[3], st));
+        g->tev_used[1] = 1;
     }
     double h = g->directed ? 1.0 : 0.5;
     // optional k-source estimator scaling (n/k, refs [3],[9]) and the
@@ -745,7 +930,7 @@ static int single_source_impl(bc_graph *g, int32_t s, int32_t *d, double *sigma,
     if (e == cudaSuccess) e = cudaMemsetAsync(dbc, 0, n * sizeof(double), g->stream);
     if (e == cudaSuccess) e = cudaMemsetAsync(dn, 0, sizeof(int), g->stream);
     if (e == cudaSuccess) e = cudaMemcpyAsync(dsrc, &s, sizeof(int), cudaMemcpyHostToDevice, g->stream);
-    if (e == cudaSuccess) e = cudaMemsetAsync(g->counters, 0, 2 * sizeof(unsigned long long), g->stream);
+    if (e == cudaSuccess) e = cudaMemsetAsync(g->counters, 0, 3 * sizeof(unsigned long long), g->stream);
     DevStats *dst = nullptr;
     if (e == cudaSuccess) e = cudaMalloc(&dst, sizeof(DevStats));
     if (e == cudaSuccess) e = cudaMemsetAsync(dst, 0, sizeof(DevStats), g->stream);
@@ -830,6 +1015,89 @@ extern "C" int bc_trace_source(bc_graph *g, int32_t s, int32_t *level_sizes, int
                               level_sizes, fwd_cycles, bwd_cycles);
 }
 
+extern "C" int bc_batch_sources(bc_graph *g, const int32_t *sources, int32_t k, int32_t *d, double *sigma,
+                                double *delta) {
+    if (!g || !sources) return fail(BC_EINVAL, "NULL argument");
+    if (g->directed) return fail(BC_EINVAL, "the batched engine needs an undirected graph");
+    if (k < 1 || k > bcbatch::BW) return fail(BC_EINVAL, "k=%d outside 1..64", k);
+    for (int i = 0; i < k; ++i)
+        if (sources[i] < 0 || sources[i] >= g->n) return fail(BC_EINVAL, "sources[%d]=%d out of range", i, sources[i]);
+    DeviceGuard dg(g->device);
+    CK(cudaEventSynchronize(g->done));
+    int rc = alloc_batch(g, k);
+    if (rc) return rc;
+    const size_t n = (size_t)g->n, kn = (size_t)k * n;
+    int *dsrc = nullptr, *dd = nullptr;
+    double *ds = nullptr, *ddel = nullptr, *dbc = nullptr;
+    DevStats *dst = nullptr;
+    cudaError_t e = cudaMalloc(&dsrc, (size_t)k * sizeof(int));
+    if (e == cudaSuccess) e = cudaMalloc(&dd, kn * sizeof(int));
+    if (e == cudaSuccess) e = cudaMalloc(&ds, kn * sizeof(double));
+    if (e == cudaSuccess) e = cudaMalloc(&ddel, kn * sizeof(double));
+    if (e == cudaSuccess) e = cudaMalloc(&dbc, n * sizeof(double));
+    if (e == cudaSuccess) e = cudaMalloc(&dst, sizeof(DevStats));
+    if (e == cudaSuccess) e = cudaMemcpy(dsrc, sources, (size_t)k * sizeof(int), cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemset(dd, 0xFF, kn * sizeof(int));
+    if (e == cudaSuccess) e = cudaMemset(ds, 0, kn * sizeof(double));
+    if (e == cudaSuccess) e = cudaMemset(ddel, 0, kn * sizeof(double));
+    if (e == cudaSuccess) e = cudaMemset(dbc, 0, n * sizeof(double));
+    if (e == cudaSuccess) e = cudaMemset(dst, 0, sizeof(DevStats));
+    if (e == cudaSuccess) e = cudaMemset(g->bt.ovf_n, 0, sizeof(long long));
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();  // the launch stream does not wait on memsets
+    if (e != cudaSuccess) rc = fail(e == cudaErrorMemoryAllocation ? BC_ENOMEM : BC_ECUDA, "%s", cudaGetErrorString(e));
+    if (rc == BC_OK) {
+        bcbatch::BParams bp = batch_params(g, dsrc, 0, k, dbc);
+        bp.stats = dst;
+        bp.dbg_d = dd;
+        bp.dbg_sigma = ds;
+        bp.dbg_delta = ddel;
+        const int saved = g->launches, saved_bc = g->bc_launches, saved_ran = g->batch_ran;
+        rc = launch_batch(g, bp, g->stream);
+        g->launches = saved;
+        g->bc_launches = saved_bc;
+        g->batch_ran = saved_ran;
+    }
+    if (rc == BC_OK) {
+        long long novf = 0;
+        e = cudaStreamSynchronize(g->stream);
+        if (e == cudaSuccess) e = cudaMemcpy(&novf, g->bt.ovf_n, sizeof(long long), cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) rc = fail(BC_ECUDA, "%s", cudaGetErrorString(e));
+        else if (novf) rc = fail(BC_EINVAL, "batch deeper than batch_levels=%d", g->bt.Lcap);
+    }
+    if (rc == BC_OK) {
+        // rows are in internal ids: gather back to the caller's ids
+        std::vector<char> tmp(n * sizeof(double));
+        auto fetch = [&](void *host, const void *dev, size_t elem) -> cudaError_t {
+            if (!host) return cudaSuccess;
+            for (int b = 0; b < k; ++b) {
+                char *h = static_cast<char *>(host) + (size_t)b * n * elem;
+                const char *dv = static_cast<const char *>(dev) + (size_t)b * n * elem;
+                if (!g->perm) {
+                    cudaError_t r = cudaMemcpy(h, dv, n * elem, cudaMemcpyDeviceToHost);
+                    if (r != cudaSuccess) return r;
+                    continue;
+                }
+                cudaError_t r = cudaMemcpy(tmp.data(), dv, n * elem, cudaMemcpyDeviceToHost);
+                if (r != cudaSuccess) return r;
+                for (size_t v = 0; v < n; ++v) memcpy(h + v * elem, tmp.data() + (size_t)g->h_perm[v] * elem, elem);
+            }
+            return cudaSuccess;
+        };
+        e = fetch(d, dd, sizeof(int));
+        if (e == cudaSuccess) e = fetch(sigma, ds, sizeof(double));
+        if (e == cudaSuccess) e = fetch(delta, ddel, sizeof(double));
+        if (e != cudaSuccess) rc = fail(BC_ECUDA, "%s", cudaGetErrorString(e));
+    }
+    cudaFree(dsrc);
+    cudaFree(dd);
+    cudaFree(ds);
+    cudaFree(ddel);
+    cudaFree(dbc);
+    cudaFree(dst);
+    if (rc == BC_OK) g_err[0] = 0;
+    return rc;
+}
+
 extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {
     if (!g || !st) return fail(BC_EINVAL, "NULL argument");
     DeviceGuard dg(g->device);
@@ -853,6 +1121,8 @@ extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {
     st->kernel_launches = g->launches;
     st->bc_kernel_launches = g->bc_launches;
     for (int q = 0; q < 4; ++q) st->phase_cycles[q] = (int64_t)h.phase_cycles[q];
+    st->batches = (int64_t)h.batches;
+    st->batch_overflows = (int64_t)h.batch_overflows;
     st->kernel_ms = 0.0;
     for (int i = 0; i < 2; ++i)
         if (g->tev_used[i]) {

@@ -1,0 +1,72 @@
+// bc_batch.cuh -- multi-source batched engine: 64 sources per batch, level-synchronous
+// over the whole GPU (cooperative persistent kernel, one grid barrier per level).
+//
+// The same per-source Brandes computation as bc_kernel (Alg. 1-3; d, sigma,
+// delta of every source are unchanged), scheduled differently: source b of a batch owns
+// bit b of a 64-bit mask per vertex and level, F_L[v] = { b : d_b(v) = L }.  A vertex v
+// is expanded once per level L at which ANY source of the batch has it (the union of the
+// 64 frontiers), so each CSR row read serves every source that has v at that level
+// (Kepler-era design expanded it once per source).  Warp lanes map to
+// sources (lane l owns sources l and l+32), so the sigma / omega gathers of one arc are
+// one coalesced 512-byte row of a vertex-major [n][64] fp64 array.
+//
+//   forward level L, u in Q_L, f = F_L[u], for x in N(u) (CSR order):
+//     sigma pull (Alg. 2 l.7-8 as a pull, R18): b in f & F_{L-1}[x] -> acc_b += sigma_b(x)
+//     discovery  (Alg. 2 l.5-6): b in f & ~(F_{L-1} | F_L | F_{L+1})[x] -> F_{L+1}[x] |= b
+//       (undirected: every neighbour of a level-L vertex is on L-1, L or L+1, so these
+//        three masks are the whole "visited" test), x enqueued into Q_{L+1} once
+//   backward level L (Alg. 3, omega trick): b in f & F_{L+1}[x] -> acc_b += omega_b(x),
+//     delta_b(u) = sigma_b(u) * acc_b, omega_b(u) = (1 + delta_b(u)) / sigma_b(u),
+//     bc[u] += sum_b delta_b(u)  (Eq. 3)
+//
+// Rows longer than CH arcs ("hubs") are split into CH-arc chunks spread over the grid;
+// their partial sums meet in hacc and are finished after one more grid barrier.
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace bcdev {
+struct DevStats;
+}
+
+namespace bcbatch {
+
+constexpr int BW = 64;        // sources per batch (bits of a mask word)
+constexpr int MAX_LCAP = 254; // level slabs per vertex = Lcap + 2 <= 256
+
+struct BParams {
+    int n;
+    const int *__restrict__ ro;   // int32 CSR (internal ids)
+    const int *__restrict__ col;
+    const int *sources;           // caller ids; NULL: source = src_base + idx
+    const int *perm;              // caller id -> internal id (NULL: identity)
+    long long src_base, k;        // this launch's sources: [src_base, src_base + k) of the list
+    int Lcap;                     // levels 0..Lcap can be expanded; deeper => overflow
+    int LS;                       // Lcap + 2: mask words per vertex (vertex-major F)
+    int CH;                       // hub chunk length (arcs); rows with deg > CH are split
+    unsigned long long *F;        // F[v * LS + L] (zero between batches)
+    double *sig;                  // sig[v * 64 + b]: sigma_b(v), then omega_b(v) in place
+    int *Q;                       // union frontiers, level after level; capacity qcap
+    long long qcap;
+    int *qcnt;                    // [LS] entries per level
+    unsigned long long *hcnt;     // [LS] hub entries per level, packed (count << 40 | chunks)
+    int *grab, *hgrab;            // [LS] work counters (vertices / hub chunks)
+    unsigned long long *lvor;     // [LS] OR of the level's masks (levels statistic)
+    int *hv, *hb;                 // hub entries: vertex, first chunk index within its level
+    double *hacc;                 // [hcap][64] hub partial sums (zero between uses)
+    long long hcap;
+    double *bc;                   // BC in internal ids (accumulated with atomics)
+    bcdev::DevStats *stats;
+    const int *sampled_flag;      // non-NULL: run only if *sampled_flag == 1 (Alg. 5 EP run)
+    int *ovf_src;                 // sources of batches that exceeded Lcap (caller ids)
+    long long *ovf_n;
+    // debug export of one launch (<= 64 sources), internal ids, [64][n]; may be NULL
+    int *dbg_d;
+    double *dbg_sigma, *dbg_delta;
+};
+
+// Kernel symbol for a block size (128, 256 or 512 threads); launched cooperatively.
+const void *batch_kernel_fn(int nt);
+
+}  // namespace bcbatch

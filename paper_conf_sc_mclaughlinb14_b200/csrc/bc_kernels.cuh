@@ -48,6 +48,7 @@ struct DevStats {
     int sampling_ep;
     int sampling_median;
     int pad;
+    unsigned long long batches, batch_overflows;  // multi-source engine (bc_batch.cu)
 };
 
 struct KParams {
@@ -63,6 +64,8 @@ struct KParams {
     const int *__restrict__ perm;     // caller id -> internal id (NULL: identity)
     long long src_base;
     long long k;                      // sources in this launch
+    const long long *k_dev;           // non-NULL: k is read from device memory (batch overflows)
+    int skip_if_ep;                   // 1: do nothing when Alg. 5 chose EP (the batched engine runs)
     unsigned long long *work_counter;
     // workspace (slot-major)
     int *d;                           // GlobalLevels only
@@ -847,6 +850,8 @@ bc_kernel(KParams p) {
 
     Counters c;
     const int run_ep = (p.launch_mode == LM_SAMPLED && p.sampled_flag) ? *p.sampled_flag : 0;
+    if (p.skip_if_ep && run_ep) return;  // uniform over the grid
+    const long long K = p.k_dev ? *p.k_dev : p.k;
     lv.template reset_all<NT>(p.code_words);
     if (threadIdx.x == 0) {
         sm.nbig = 0;
@@ -857,7 +862,7 @@ bc_kernel(KParams p) {
         if (threadIdx.x == 0) sm.idx = (long long)atomicAdd(p.work_counter, 1ULL);
         __syncthreads();
         const long long idx = sm.idx;
-        if (idx >= p.k) break;
+        if (idx >= K) break;
         int s = p.sources ? p.sources[p.src_base + idx] : (int)(p.src_base + idx);
         if (p.perm) s = p.perm[s];  // caller's id -> internal id
         // Alg. 1; all other entries are already unvisited / zero.
