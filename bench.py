@@ -205,6 +205,8 @@ B200_EP_GUARD = 2147483647
 
 def bench_options(args):
     o = {"strategy": args.strategy}
+    if args.engine != "auto":
+        o["engine"] = args.engine
     if args.strategy == "sampling":
         o["ep_min_frontier"] = 512 if args.paper_params else int(args.ep_guard)
     return o
@@ -382,6 +384,8 @@ def main():
     ap.add_argument("--paper-params", action="store_true",
                     help="use the paper's EP guard (512) instead of the B200-retuned one")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--engine", default="auto", choices=["auto", "per_source", "batched"],
+                    help="source scheduling (include/bc.h BC_ENGINE_*)")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()

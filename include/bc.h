@@ -63,7 +63,9 @@ enum {
 enum {
     BC_ENGINE_AUTO = 0,       /* per-source engine, except that a SAMPLING run whose Alg. 5
                                  decision is EP ("small-world": median depth < gamma*log2 n)
-                                 on an undirected graph runs its main phase batched          */
+                                 on a large (n >= 2^21) undirected graph with a skewed degree
+                                 distribution runs its main phase batched (measured faster
+                                 there only)                                   */
     BC_ENGINE_PER_SOURCE = 1, /* one CTA per source (bc_kernel), every level WE or EP as the
                                  strategy chooses                                            */
     BC_ENGINE_BATCHED = 2     /* undirected graphs: 64 sources per batch, level-synchronous
@@ -109,8 +111,9 @@ typedef struct bc_options {
     int32_t engine;          /* BC_ENGINE_*, default BC_ENGINE_AUTO                            */
     int32_t batch_levels;    /* batched engine: BFS levels a batch may have (0 = auto 64, max
                                 254); sources of a deeper batch are rerun per source         */
-    int32_t hub_chunk;       /* batched engine: rows longer than this are split into chunks of
-                                this many arcs spread over the GPU (0 = auto 1024)            */
+    int32_t hub_chunk;       /* batched engine: minimum arcs per warp range when a BFS level's
+                                arcs are cut into equal warp ranges (rows of any length are
+                                split across ranges); 0 = auto 64                            */
 } bc_options;
 
 typedef struct bc_stats {

@@ -115,11 +115,11 @@ struct bc_graph {
     std::vector<int> h_ro;              // internal CSR offsets (hub counts for any chunk size)
     struct Batch {
         int ready = 0, failed = 0;
-        int Lcap = 0, LS = 0, CH = 0, nt = 256, grid = 0;
-        long long qcap = 0, hcap = 0;
-        unsigned long long *F = nullptr, *hcnt = nullptr, *lvor = nullptr;
-        double *sig = nullptr, *hacc = nullptr;
-        int *Q = nullptr, *qcnt = nullptr, *grab = nullptr, *hv = nullptr, *hb = nullptr;
+        int Lcap = 0, LS = 0, nt = 256, grid = 0, nwarps = 0;
+        long long qcap = 0;
+        unsigned long long *F = nullptr, *qctr = nullptr, *lvor = nullptr;
+        double *sig = nullptr, *dacc = nullptr;
+        int *Q = nullptr, *qoff = nullptr;
         int *ovf_src = nullptr;
         long long ovf_cap = 0;
         long long *ovf_n = nullptr;
@@ -315,76 +315,71 @@ static int alloc_workspace(bc_graph *g) {
 static void free_batch(bc_graph *g) {
     bc_graph::Batch &b = g->bt;
     cudaFree(b.F);
-    cudaFree(b.hcnt);
+    cudaFree(b.qctr);
     cudaFree(b.lvor);
     cudaFree(b.sig);
-    cudaFree(b.hacc);
+    cudaFree(b.dacc);
     cudaFree(b.Q);
-    cudaFree(b.qcnt);
-    cudaFree(b.grab);
-    cudaFree(b.hv);
-    cudaFree(b.hb);
+    cudaFree(b.qoff);
     cudaFree(b.ovf_src);
     cudaFree(b.ovf_n);
     b = bc_graph::Batch{};
 }
 
 // Workspace of the batched engine: vertex-major level masks F[(Lcap + 2) n], sigma/omega
-// [n][64], the union-frontier lists Q (a vertex is in at most min(64, Lcap + 2) of them),
-// hub entries and their partial sums.  Sized on first use; ~1.3 KB per vertex at Lcap 64.
+// and accumulators [n][64], the union-frontier lists Q + their arc offsets (a vertex is
+// in at most min(64, Lcap + 2) of them).  ~2 KB per vertex at Lcap 64.
 static int alloc_batch(bc_graph *g, long long max_sources) {
     bc_graph::Batch &b = g->bt;
     const int Lcap = g->opt.batch_levels > 0 ? g->opt.batch_levels : 64;
-    const int CH = g->opt.hub_chunk > 0 ? g->opt.hub_chunk : 1024;
     const long long ovf_need = std::max<long long>(max_sources, 64);
-    if (b.ready && b.Lcap == Lcap && b.CH == CH && b.ovf_cap >= ovf_need) return BC_OK;
+    if (b.ready && b.Lcap == Lcap && b.ovf_cap >= ovf_need) return BC_OK;
     free_batch(g);
+    if ((long long)g->n >= (1LL << 24)) return fail(BC_EINVAL, "batched engine: n must be < 2^24");
     const size_t n = (size_t)std::max(g->n, 1);
     b.Lcap = Lcap;
     b.LS = Lcap + 2;
-    b.CH = CH;
-    long long nhub = 0;
-    for (int v = 0; v < g->n; ++v) nhub += (g->h_ro[v + 1] - g->h_ro[v]) > CH;
     const long long per_v = std::min(bcbatch::BW, b.LS);
     b.qcap = (long long)n * per_v;
-    b.hcap = std::max<long long>(1, nhub * per_v);
     b.ovf_cap = ovf_need;
-    CK(cudaMalloc(&b.F, n * (size_t)b.LS * 8));
-    CK(cudaMalloc(&b.sig, n * bcbatch::BW * sizeof(double)));
-    CK(cudaMalloc(&b.Q, (size_t)b.qcap * sizeof(int)));
-    CK(cudaMalloc(&b.qcnt, (size_t)b.LS * sizeof(int)));
-    CK(cudaMalloc(&b.hcnt, (size_t)b.LS * 8));
-    CK(cudaMalloc(&b.grab, 4 * (size_t)b.LS * sizeof(int)));
-    CK(cudaMalloc(&b.lvor, (size_t)b.LS * 8));
-    CK(cudaMalloc(&b.hv, (size_t)b.hcap * sizeof(int)));
-    CK(cudaMalloc(&b.hb, (size_t)b.hcap * sizeof(int)));
-    CK(cudaMalloc(&b.hacc, (size_t)b.hcap * bcbatch::BW * sizeof(double)));
-    CK(cudaMalloc(&b.ovf_src, (size_t)b.ovf_cap * sizeof(int)));
-    CK(cudaMalloc(&b.ovf_n, sizeof(long long)));
-    CK(cudaMemset(b.F, 0, n * (size_t)b.LS * 8));
-    CK(cudaMemset(b.qcnt, 0, (size_t)b.LS * sizeof(int)));
-    CK(cudaMemset(b.hcnt, 0, (size_t)b.LS * 8));
-    CK(cudaMemset(b.grab, 0, 4 * (size_t)b.LS * sizeof(int)));
-    CK(cudaMemset(b.lvor, 0, (size_t)b.LS * 8));
-    CK(cudaMemset(b.hacc, 0, (size_t)b.hcap * bcbatch::BW * sizeof(double)));
-    CK(cudaMemset(b.ovf_n, 0, sizeof(long long)));
     b.nt = 256;
     const void *fn = bcbatch::batch_kernel_fn(b.nt);
     int per_sm = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, b.nt, 0));
     if (per_sm < 1) return fail(BC_EINTERNAL, "batched kernel cannot be resident");
     b.grid = per_sm * g->num_sms;
+    b.nwarps = b.grid * b.nt / 32;
+    CK(cudaMalloc(&b.F, n * (size_t)b.LS * 8));
+    const size_t sn = (n + 31) & ~(size_t)31;
+    CK(cudaMalloc(&b.sig, sn * bcbatch::BW * sizeof(double)));
+    CK(cudaMalloc(&b.Q, (size_t)b.qcap * sizeof(int)));
+    CK(cudaMalloc(&b.qoff, (size_t)b.qcap * sizeof(int)));
+    CK(cudaMalloc(&b.qctr, (size_t)b.LS * 8));
+    CK(cudaMalloc(&b.lvor, (size_t)b.LS * 8));
+    CK(cudaMalloc(&b.dacc, sn * bcbatch::BW * sizeof(double)));
+    CK(cudaMalloc(&b.ovf_src, (size_t)b.ovf_cap * sizeof(int)));
+    CK(cudaMalloc(&b.ovf_n, sizeof(long long)));
+    CK(cudaMemset(b.F, 0, n * (size_t)b.LS * 8));
+    CK(cudaMemset(b.qctr, 0, (size_t)b.LS * 8));
+    CK(cudaMemset(b.lvor, 0, (size_t)b.LS * 8));
+    CK(cudaMemset(b.ovf_n, 0, sizeof(long long)));
     CK(cudaDeviceSynchronize());
     b.ready = 1;
     return BC_OK;
 }
 
 // Whether this call may run the batched engine (undirected graphs only: the
-// three-mask visited test relies on neighbours being on adjacent levels).
+// three-mask visited test relies on neighbours being on adjacent levels).  Auto mode
+// follows the engine comparison of DESIGN.md §7 (tools/cmp_engines.sh): the batched
+// engine wins only where the per-source state of the in-flight sources (24 B x n each)
+// is far beyond L2 AND the degree distribution is skewed (relabelled graphs: c5k
+// 1.26x), loses on c4 (n = 2^18), on the unskewed small world c5ws and on every
+// high-diameter graph; the device-side Alg. 5 flag still has to say EP.
 static bool batch_wanted(const bc_graph *g) {
     if (g->directed || g->n == 0) return false;
     if (g->opt.engine == BC_ENGINE_BATCHED) return true;
-    return g->opt.engine == BC_ENGINE_AUTO && g->opt.strategy == BC_STRATEGY_SAMPLING;
+    return g->opt.engine == BC_ENGINE_AUTO && g->opt.strategy == BC_STRATEGY_SAMPLING &&
+           g->perm != nullptr && g->n >= (1 << 21);
 }
 
 static int launch_batch(bc_graph *g, const bcbatch::BParams &bp0, cudaStream_t st) {
@@ -407,7 +402,34 @@ static int launch_batch(bc_graph *g, const bcbatch::BParams &bp0, cudaStream_t s
     }
     lc.attrs = attr;
     lc.numAttrs = na;
+    // BC_BATCH_TRACE=1: per-level cycle trace of the launch's first batch on stderr
+    // (debug tooling; synchronises the stream)
+    const char *tr = getenv("BC_BATCH_TRACE");
+    long long *dtrace = nullptr;
+    const size_t ntr = 2 * (size_t)g->bt.LS * 12;
+    if (tr && *tr == '1') {
+        CK(cudaMalloc(&dtrace, ntr * sizeof(long long)));
+        CK(cudaMemsetAsync(dtrace, 0, ntr * sizeof(long long), st));
+        bp.trace = dtrace;
+    }
     CK(cudaLaunchKernelExC(&lc, bcbatch::batch_kernel_fn(g->bt.nt), args));
+    if (dtrace) {
+        std::vector<long long> h(ntr);
+        CK(cudaMemcpyAsync(h.data(), dtrace, ntr * sizeof(long long), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        cudaFree(dtrace);
+        const int nw = g->bt.nwarps;
+        for (int dir = 0; dir < 2; ++dir)
+            for (int L = 0; L < g->bt.LS; ++L) {
+                const long long *t = &h[((size_t)dir * g->bt.LS + L) * 12];
+                if (!t[0] && !t[1]) continue;
+                fprintf(stderr, "[trace] %s L=%2d arcs=%9lld wall=%9lld maxwarp=%9lld meanwarp=%9.0f | "
+                        "rowwin %lld x %.0f cyc, pairwin %lld x %.0f cyc, pairs %lld, range %.0f cyc/warp\n",
+                        dir ? "bwd" : "fwd", L, t[3], t[0], t[1], (double)t[2] / nw,
+                        t[6], t[6] ? (double)t[4] / t[6] : 0.0, t[7], t[7] ? (double)t[5] / t[7] : 0.0, t[8],
+                        (double)t[9] / nw);
+            }
+    }
     g->launches++;
     g->bc_launches++;
     g->batch_ran = 1;
@@ -429,19 +451,16 @@ static bcbatch::BParams batch_params(bc_graph *g, const int *d_sources, long lon
     bp.k = k;
     bp.Lcap = b.Lcap;
     bp.LS = b.LS;
-    bp.CH = b.CH;
+    bp.min_range = g->opt.hub_chunk > 0 ? g->opt.hub_chunk : 64;
     bp.F = b.F;
     bp.sig = b.sig;
     bp.Q = b.Q;
+    bp.qoff = b.qoff;
     bp.qcap = b.qcap;
-    bp.qcnt = b.qcnt;
-    bp.hcnt = b.hcnt;
-    bp.grab = b.grab;
+    bp.qctr = b.qctr;
     bp.lvor = b.lvor;
-    bp.hv = b.hv;
-    bp.hb = b.hb;
-    bp.hacc = b.hacc;
-    bp.hcap = b.hcap;
+    bp.dacc = b.dacc;
+    bp.sn = ((size_t)std::max(g->n, 1) + 31) & ~(size_t)31;
     bp.bc = acc_bc;
     bp.stats = g->stats;
     bp.ovf_src = b.ovf_src;

@@ -1,8 +1,9 @@
 // bc_batch.cu -- the multi-source batched engine (design in bc_batch.cuh).
 //
 // One cooperative persistent kernel; all CTAs work on one batch of 64 sources at a time
-// and meet at a grid barrier after every level.  Work inside a level is pulled from
-// global counters (16 frontier vertices, or one hub chunk, per grab) by whole warps.
+// and meet at a grid barrier after every level.  Inside a level every warp owns an equal
+// contiguous range of the level's arc space (merge-path style), so rows of any degree --
+// hubs included -- are spread evenly and no warp is a long pole.
 #define BC_INSTANCE_TU
 #include "bc_kernels.cuh"
 #include "bc_batch.cuh"
@@ -17,149 +18,21 @@ using bcdev::DevStats;
 using bcdev::FULL;
 using bcdev::TWO53;
 
-constexpr int GRAB = 16;                          // frontier vertices per warp grab
-constexpr unsigned long long CNT_ONE = 1ull << 40; // packed hub counter: count << 40 | chunks
-constexpr unsigned long long CH_MASK = CNT_ONE - 1;
+constexpr unsigned long long CNT_ONE = 1ull << 40;  // packed level counter: entries << 40 | arcs
+constexpr unsigned long long ARC_MASK = CNT_ONE - 1;
+constexpr int BIG = 0x7FFFFFFF;
 
-struct Cnt {
-    unsigned long long reached = 0, ar = 0, dag = 0, sc = 0;
+// sigma / acc layout: vertex-major, entry (b, v) at v * 64 + b (the pairs of one vertex
+// share sectors: measured 2x faster on c4 than source-major b * sn + v)
+__device__ __forceinline__ size_t sidx(const BParams &, int b, int v) { return (size_t)v * BW + (size_t)b; }
+
+struct Cnt {  // per-lane counters of one batch (32-bit: a batch is ~10^8 events per warp at most)
+    unsigned reached = 0, ar = 0, dag = 0, sc = 0;
     int inexact = 0;
 };
 
 __device__ __forceinline__ unsigned long long shfl64(unsigned long long v, int src) {
     return __shfl_sync(FULL, v, src);
-}
-
-// Append hub vertex x (deg > CH) to the hub list of level `lvl` (entries start at hlo).
-__device__ __forceinline__ void hub_push(const BParams &p, int lvl, int hlo, int x, int deg) {
-    const unsigned long long nch = (unsigned long long)((deg + p.CH - 1) / p.CH);
-    const unsigned long long old = atomicAdd(&p.hcnt[lvl], CNT_ONE | nch);
-    const int pos = hlo + (int)(old >> 40);
-    p.hv[pos] = x;
-    p.hb[pos] = (int)(old & CH_MASK);
-}
-
-// Sum over the arcs j (in ascending lane order = CSR order) of the current 32-arc
-// group whose mask bit of this lane's source is set: acc0 += val[x_j*64 + lane],
-// acc1 += val[x_j*64 + 32 + lane].  Four arcs' gathers are issued before they are
-// added; skipped slots add +0.0, which leaves the sums bit-identical.
-__device__ __forceinline__ void gather_group(const double *__restrict__ val, int x, unsigned long long m,
-                                             int lane, double &acc0, double &acc1) {
-    unsigned sel = __ballot_sync(FULL, m != 0ull);
-    while (sel) {
-        int j[4];
-#pragma unroll
-        for (int t = 0; t < 4; ++t) {
-            j[t] = sel ? __ffs(sel) - 1 : -1;
-            sel &= sel - 1u;  // sel == 0 stays 0
-        }
-        double g0[4], g1[4];
-#pragma unroll
-        for (int t = 0; t < 4; ++t) {
-            const int jj = j[t] < 0 ? 0 : j[t];
-            const int xj = __shfl_sync(FULL, x, jj);
-            const unsigned long long mj = j[t] < 0 ? 0ull : shfl64(m, jj);
-            const double *row = val + (size_t)xj * BW;
-            g0[t] = (mj >> lane) & 1ull ? __ldcg(row + lane) : 0.0;
-            g1[t] = (mj >> (lane + 32)) & 1ull ? __ldcg(row + 32 + lane) : 0.0;
-        }
-#pragma unroll
-        for (int t = 0; t < 4; ++t) {
-            acc0 += g0[t];
-            acc1 += g1[t];
-        }
-    }
-}
-
-// Forward scan of arcs [a0, a1) of a level-L vertex with source mask f (one warp).
-template <bool PULL>
-__device__ __forceinline__ void fwd_seg(const BParams &p, int L, unsigned long long f, int a0, int a1,
-                                        int qlo_next, int hlo_next, double &acc0, double &acc1, Cnt &c) {
-    const int lane = threadIdx.x & 31;
-    const int LS = p.LS;
-    for (int base = a0; base < a1; base += 32) {
-        const int a = base + lane;
-        const bool ok = a < a1;
-        const int x = ok ? __ldg(&p.col[a]) : 0;
-        unsigned long long fp = 0ull, fc = 0ull, fn = 0ull;
-        unsigned long long *Fx = p.F + (size_t)x * LS + L;
-        if (ok) {
-            if (PULL) fp = __ldcg(Fx - 1);
-            fc = __ldcg(Fx);
-            fn = __ldcg(Fx + 1);
-        }
-        const unsigned long long pm = f & fp;
-        const unsigned long long dm = ok ? (f & ~(fp | fc | fn)) : 0ull;
-        bool fresh = false;
-        if (dm) fresh = atomicOr(Fx + 1, dm) == 0ull;  // first discoverer enqueues x
-        const unsigned nb = __ballot_sync(FULL, fresh);
-        if (nb) {
-            const int leader = __ffs(nb) - 1;
-            int qb = 0;
-            if (lane == leader) qb = atomicAdd(&p.qcnt[L + 1], __popc(nb));
-            qb = __shfl_sync(FULL, qb, leader);
-            if (fresh) {
-                p.Q[qlo_next + qb + __popc(nb & ((1u << lane) - 1u))] = x;
-                const int deg = __ldg(&p.ro[x + 1]) - __ldg(&p.ro[x]);
-                if (deg > p.CH) hub_push(p, L + 1, hlo_next, x, deg);
-            }
-        }
-        if (PULL) {
-            c.dag += (unsigned long long)__popcll(pm);
-            gather_group(p.sig, x, pm, lane, acc0, acc1);
-        }
-    }
-}
-
-// Backward scan of arcs [a0, a1) of a level-L vertex: omega of successors (F_{L+1}).
-__device__ __forceinline__ void bwd_seg(const BParams &p, int L, unsigned long long f, int a0, int a1,
-                                        double &acc0, double &acc1) {
-    const int lane = threadIdx.x & 31;
-    for (int base = a0; base < a1; base += 32) {
-        const int a = base + lane;
-        const bool ok = a < a1;
-        const int x = ok ? __ldg(&p.col[a]) : 0;
-        const unsigned long long fs = ok ? __ldcg(p.F + (size_t)x * p.LS + L + 1) : 0ull;
-        gather_group(p.sig, x, f & fs, lane, acc0, acc1);
-    }
-}
-
-// Alg. 3 l.8 with the omega trick for the lane's two sources of vertex u (mask f),
-// then Eq. 3: returns the lane's share of sum_b delta_b(u).
-__device__ __forceinline__ double finish_pair(const BParams &p, int u, unsigned long long f, double acc0,
-                                              double acc1) {
-    const int lane = threadIdx.x & 31;
-    double bs = 0.0;
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-        const int b = lane + 32 * h;
-        if ((f >> b) & 1ull) {
-            double *e = p.sig + (size_t)u * BW + b;
-            const double su = __ldcg(e);
-            const double delta = su * (h ? acc1 : acc0);
-            *e = (1.0 + delta) / su;
-            bs += delta;
-            if (p.dbg_delta) p.dbg_delta[(size_t)b * p.n + u] = delta;
-        }
-    }
-    return bs;
-}
-
-__device__ __forceinline__ void store_sigma(const BParams &p, int u, int L, unsigned long long f, double acc0,
-                                            double acc1) {
-    const int lane = threadIdx.x & 31;
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-        const int b = lane + 32 * h;
-        if ((f >> b) & 1ull) {
-            const double s = h ? acc1 : acc0;
-            p.sig[(size_t)u * BW + b] = s;
-            if (p.dbg_d) {
-                p.dbg_d[(size_t)b * p.n + u] = L;
-                p.dbg_sigma[(size_t)b * p.n + u] = s;
-            }
-        }
-    }
 }
 
 __device__ __forceinline__ double warp_sum(double v) {
@@ -168,274 +41,497 @@ __device__ __forceinline__ double warp_sum(double v) {
     return v;
 }
 
-// Hub entry holding chunk ci of a level: the last entry in [hlo, hlo + hn) whose first
-// chunk index is <= ci (first-chunk indices grow with the entry index).
-__device__ __forceinline__ int hub_find(const BParams &p, int hlo, int hn, int ci) {
-    int lo = 0, hi = hn - 1;
-    while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (__ldcg(&p.hb[hlo + mid]) <= ci) lo = mid;
-        else hi = mid - 1;
+// Rows r0 .. r0+31 of the current level, lane j holding row r0 + j.
+struct Rows {
+    int r0;
+    int u;                 // vertex
+    unsigned long long f;  // its source mask at this level
+    int cbeg;              // CSR position of level arc a of this row = a + cbeg
+    int start, nxt;        // the row's arcs [start, nxt) in the level's arc space
+};
+
+__device__ __forceinline__ void load_rows(const BParams &p, Rows &R, int r0, int qlo, int qn, int A, int L) {
+    const int r = r0 + (threadIdx.x & 31);
+    R.r0 = r0;
+    if (r < qn) {
+        R.u = __ldcg(&p.Q[qlo + r]);
+        R.start = __ldcg(&p.qoff[qlo + r]);
+        R.nxt = r + 1 < qn ? __ldcg(&p.qoff[qlo + r + 1]) : A;
+        R.f = __ldcg(&p.F[(size_t)R.u * p.LS + L]);
+        R.cbeg = __ldg(&p.ro[R.u]) - R.start;
+    } else {
+        R.u = 0;
+        R.start = R.nxt = BIG;
+        R.f = 0ull;
+        R.cbeg = 0;
     }
-    return hlo + lo;
+}
+
+// Largest r in [0, qn) with qoff[qlo + r] <= a (32-ary search by the whole warp).
+__device__ __forceinline__ int find_row(const BParams &p, int qlo, int qn, int a) {
+    const int lane = threadIdx.x & 31;
+    int lo = 0, hi = qn;
+    while (hi - lo > 32) {
+        const int step = (hi - lo + 31) >> 5;
+        const int q = lo + lane * step;
+        const int v = q < hi ? __ldcg(&p.qoff[qlo + q]) : BIG;
+        const int c = __popc(__ballot_sync(FULL, v <= a));
+        lo += (c - 1) * step;
+        hi = min(hi, lo + step);
+    }
+    const int q = lo + lane;
+    const int v = q < hi ? __ldcg(&p.qoff[qlo + q]) : BIG;
+    return lo + __popc(__ballot_sync(FULL, v <= a)) - 1;
+}
+
+struct Level {
+    int L, qlo, qn, A, qlo_next;
+    int per;  // arcs per warp range
+};
+
+// Window inside one long row (lanes = sources): the row's pairs are dense (a hub at its
+// usual level), so each arc's gathers are two coalesced warp loads, summed in arc order
+// in registers and reduced once per window -- per-pair reductions would all hit the same
+// 64 accumulators.  Four arcs' gathers are issued before they are added.
+template <bool FWD>
+__device__ __forceinline__ void gather_row_window(const BParams &p, int x, unsigned long long m, int u) {
+    constexpr int U = FWD ? 8 : 4;  // arcs per round: 2U (fwd) / 4U (bwd) loads in flight per lane
+    const int lane = threadIdx.x & 31;
+    double acc0 = 0.0, acc1 = 0.0;
+    unsigned sel = __ballot_sync(FULL, m != 0ull);
+    while (sel) {
+        double s0[U], s1[U], a0[U], a1[U];
+        bool h0[U], h1[U];
+#pragma unroll
+        for (int t = 0; t < U; ++t) {  // all loads of the round first ...
+            const int j = sel ? __ffs(sel) - 1 : -1;
+            sel &= sel - 1u;
+            const int xj = __shfl_sync(FULL, x, j < 0 ? 0 : j);
+            const unsigned long long mj = shfl64(m, j < 0 ? 0 : j);
+            h0[t] = j >= 0 && ((mj >> lane) & 1ull);
+            h1[t] = j >= 0 && ((mj >> (lane + 32)) & 1ull);
+            const size_t r0 = sidx(p, lane, xj), r1 = sidx(p, lane + 32, xj);
+            s0[t] = h0[t] ? __ldca(p.sig + r0) : 1.0;
+            s1[t] = h1[t] ? __ldca(p.sig + r1) : 1.0;
+            if (!FWD) {
+                a0[t] = h0[t] ? __ldca(p.dacc + r0) : 0.0;
+                a1[t] = h1[t] ? __ldca(p.dacc + r1) : 0.0;
+            }
+        }
+#pragma unroll
+        for (int t = 0; t < U; ++t) {  // ... then the arithmetic, in arc order
+            if (FWD) {
+                acc0 += h0[t] ? s0[t] : 0.0;
+                acc1 += h1[t] ? s1[t] : 0.0;
+            } else {  // omega_b(x) = 1 / sigma_b(x) + acc_b(x)
+                acc0 += h0[t] ? 1.0 / s0[t] + a0[t] : 0.0;
+                acc1 += h1[t] ? 1.0 / s1[t] + a1[t] : 0.0;
+            }
+        }
+    }
+    double *tgt = FWD ? p.sig : p.dacc;
+    if (acc0 != 0.0) atomicAdd(tgt + sidx(p, lane, u), acc0);
+    if (acc1 != 0.0) atomicAdd(tgt + sidx(p, lane + 32, u), acc1);
+}
+
+// Window spanning several rows (lanes = arcs): the window's (arc, source) pairs are
+// compacted into a per-warp list in shared memory and dealt out evenly, U pairs per
+// lane in flight: gathers first, then fire-and-forget fp64 reductions into the row's
+// accumulator (sums of integers < 2^53 are exact in any order).
+template <bool FWD>
+__device__ __forceinline__ void accumulate_pairs(const BParams &p, uint16_t *lst, int x, int u,
+                                                 unsigned long long m) {
+    constexpr int U = FWD ? 6 : 4;
+    const int lane = threadIdx.x & 31;
+    const int c = __popcll(m);
+    int incl = c;
+#pragma unroll
+    for (int s = 1; s < 32; s <<= 1) {
+        const int y = __shfl_up_sync(FULL, incl, s);
+        if (lane >= s) incl += y;
+    }
+    const int P = __shfl_sync(FULL, incl, 31);
+    int k = incl - c;
+    while (m) {
+        const int b = __ffsll((long long)m) - 1;
+        m &= m - 1ull;
+        lst[k++] = (uint16_t)((lane << 6) | b);
+    }
+    __syncwarp();
+    for (int k0 = 0; k0 < P; k0 += 32 * U) {
+        int bb[U], uu[U];
+        double sv[U], av[U];
+#pragma unroll
+        for (int t = 0; t < U; ++t) {
+            const int kk = k0 + t * 32 + lane;
+            const int e = kk < P ? lst[kk] : -1;
+            const int j = e < 0 ? 0 : e >> 6;
+            const int xj = __shfl_sync(FULL, x, j);
+            uu[t] = __shfl_sync(FULL, u, j);
+            bb[t] = e < 0 ? -1 : (e & 63);
+            const size_t r = sidx(p, bb[t] < 0 ? 0 : bb[t], xj);
+            sv[t] = bb[t] >= 0 ? __ldca(p.sig + r) : 1.0;
+            if (!FWD) av[t] = bb[t] >= 0 ? __ldca(p.dacc + r) : 0.0;
+        }
+#pragma unroll
+        for (int t = 0; t < U; ++t)
+            if (bb[t] >= 0)  // RED.ADD.F64 (result unused)
+                atomicAdd((FWD ? p.sig : p.dacc) + sidx(p, bb[t], uu[t]), FWD ? sv[t] : 1.0 / sv[t] + av[t]);
+    }
+    __syncwarp();
+}
+
+// ---- one warp's range [a_lo, a_hi) of level L's arc space
+//
+// Software-pipelined: the rows of window i+1 are fetched in two stages (Q / offsets,
+// then mask / CSR start) behind window i's column, mask, discovery and gather loads,
+// and the enqueue reservation of window i is consumed only after its gathers are
+// issued, so a window costs about four dependent memory round trips.
+
+struct RowStage {  // stage 1 of a row fetch (lane j: row r0 + j)
+    int r0, u, start, nxt;
+};
+
+__device__ __forceinline__ void rows_stage1(const BParams &p, RowStage &S, int r0, int qlo, int qn, int A) {
+    const int r = r0 + (threadIdx.x & 31);
+    S.r0 = r0;
+    if (r < qn) {
+        S.u = __ldcg(&p.Q[qlo + r]);
+        S.start = __ldcg(&p.qoff[qlo + r]);
+        S.nxt = r + 1 < qn ? __ldcg(&p.qoff[qlo + r + 1]) : A;
+    } else {
+        S.u = -1;
+        S.start = S.nxt = BIG;
+    }
+}
+
+__device__ __forceinline__ void rows_stage2(const BParams &p, Rows &R, const RowStage &S, int L) {
+    R.r0 = S.r0;
+    R.u = S.u < 0 ? 0 : S.u;
+    R.start = S.start;
+    R.nxt = S.nxt;
+    if (S.u >= 0) {
+        R.f = __ldcg(&p.F[(size_t)S.u * p.LS + L]);
+        R.cbeg = __ldg(&p.ro[S.u]) - S.start;
+    } else {
+        R.f = 0ull;
+        R.cbeg = 0;
+    }
+}
+
+template <bool FWD>
+__device__ __forceinline__ void process_range(const BParams &p, const Level &lv, int a_lo, int a_hi, Cnt &c,
+                                              unsigned long long &wor, uint16_t *lst, long long *tprof) {
+    const int lane = threadIdx.x & 31;
+    const int L = lv.L;
+    const int LS = p.LS;
+    const long long tr0 = clock64();
+    int rb = find_row(p, lv.qlo, lv.qn, a_lo);  // row containing arc `base`
+    Rows R;
+    RowStage S;
+    rows_stage1(p, S, rb, lv.qlo, lv.qn, lv.A);
+    rows_stage2(p, R, S, L);
+    for (int base = a_lo; base < a_hi; base += 32) {
+        // rows ending inside the window: bit k <=> some cached row ends at arc base + k
+        const int rel = R.nxt - base;
+        const unsigned M = __reduce_or_sync(FULL, (rel >= 1 && rel <= 31) ? (1u << rel) : 0u);
+        const bool end32 = __any_sync(FULL, rel == 32);
+        const unsigned below = lane == 31 ? FULL : ((2u << lane) - 1u);
+        const int o = __popc(M & below);  // lane's row, relative to rb
+        const int a = base + lane;
+        const bool ok = a < a_hi;
+        const unsigned long long f = shfl64(R.f, o);
+        const int cb = __shfl_sync(FULL, R.cbeg, o);
+        const int u = __shfl_sync(FULL, R.u, o);
+        const int rs = __shfl_sync(FULL, R.start, o), re = __shfl_sync(FULL, R.nxt, o);
+        const int x = ok ? __ldg(&p.col[a + cb]) : 0;                 // trip 1
+        const int rb_next = rb + __popc(M) + (end32 ? 1 : 0);         // row containing arc base + 32
+        const bool more = base + 32 < a_hi;
+        const bool newrows = more && rb_next != rb;
+        if (newrows) rows_stage1(p, S, rb_next, lv.qlo, lv.qn, lv.A);  // behind trip 1
+        unsigned long long m;  // sources whose accumulator for u takes a term from x
+        unsigned nb = 0u;
+        int dv = 0, incl = 0;
+        unsigned long long resv = 0ull;
+        if (FWD) {
+            unsigned long long fp = 0ull, fc = 0ull, fn = 0ull;
+            unsigned long long *Fx = p.F + (size_t)x * LS + L;
+            if (ok) {                                                  // trip 2
+                if (L > 0) fp = __ldca(Fx - 1);  // levels L-1, L: fixed during this level
+                fc = __ldca(Fx);
+                fn = __ldcg(Fx + 1);             // level L+1: being built (atomics, L2)
+            }
+            m = f & fp;
+            const unsigned long long dm = ok ? (f & ~(fp | fc | fn)) : 0ull;
+            bool fresh = false;
+            if (dm) {                                                  // trip 3
+                dv = __ldg(&p.ro[x + 1]) - __ldg(&p.ro[x]);            // (degree, in the same trip)
+                const unsigned long long old = atomicOr(Fx + 1, dm);
+                fresh = old == 0ull;  // the first discoverer enqueues x
+                unsigned long long nw = dm & ~old;  // (x, b) pairs this lane discovered
+                while (nw) {
+                    const int b = __ffsll((long long)nw) - 1;
+                    nw &= nw - 1ull;
+                    p.sig[sidx(p, b, x)] = 0.0;
+                    p.dacc[sidx(p, b, x)] = 0.0;
+                }
+            }
+            nb = __ballot_sync(FULL, fresh);
+            if (nb) {  // reserve Q entries + arcs; the result is consumed after the gathers
+                if (!fresh) dv = 0;
+                incl = dv;
+#pragma unroll
+                for (int s = 1; s < 32; s <<= 1) {
+                    const int y = __shfl_up_sync(FULL, incl, s);
+                    if (lane >= s) incl += y;
+                }
+                const int tot = __shfl_sync(FULL, incl, 31);
+                if (lane == 0)
+                    resv = atomicAdd(&p.qctr[L + 1], ((unsigned long long)__popc(nb) << 40) | (unsigned long long)tot);
+            }
+            c.dag += (unsigned)__popcll(m);
+            if (ok && a == rs) {  // first arc of the row: per-row statistics
+                c.reached += (unsigned)__popcll(f);
+                c.ar += (unsigned)__popcll(f) * (unsigned)(re - rs);
+                wor |= f;
+            }
+        } else {
+            m = ok ? (f & __ldca(p.F + (size_t)x * LS + L + 1)) : 0ull;  // trip 2
+        }
+        if (newrows) rows_stage2(p, R, S, L);  // next window's rows (stage 1 has long arrived)
+        // one dense row (a hub at its usual level): lanes = sources, register sums;
+        // otherwise lanes = pairs.  `u_row` is the window's row when M == 0.
+        const int npairs = __reduce_add_sync(FULL, (unsigned)__popcll(m));
+        const long long tg = clock64();
+        const bool rowwin = M == 0u && npairs > 96;
+        if (rowwin) gather_row_window<FWD>(p, x, m, u);   // trip 4
+        else if (npairs) accumulate_pairs<FWD>(p, lst, x, u, m);
+        if (tprof && lane == 0) {
+            tprof[rowwin ? 0 : 1] += clock64() - tg;
+            tprof[rowwin ? 2 : 3] += 1;
+            tprof[4] += npairs;
+        }
+        if (FWD && nb) {
+            resv = shfl64(resv, 0);
+            if ((nb >> lane) & 1u) {
+                const int pos = lv.qlo_next + (int)(resv >> 40) + __popc(nb & ((1u << lane) - 1u));
+                p.Q[pos] = x;
+                p.qoff[pos] = (int)(resv & ARC_MASK) + incl - dv;
+            }
+        }
+        if (lane == 0) c.sc += (unsigned)min(32, a_hi - base);
+        rb = rb_next;
+    }
+    if (tprof && lane == 0) tprof[5] += clock64() - tr0;
+}
+
+// delta_b(u) = sigma_b(u) * acc_b(u) for every pair of level L (complete after the
+// barrier that ended backward level L), summed over b into bc[u] (Eq. 3).
+// Thread per (entry, source): 64 consecutive threads share one Q entry.
+template <int NT>
+__device__ __forceinline__ void delta_pass(const BParams &p, int L, int qlo, int qn, Cnt &c) {
+    const int gtid = blockIdx.x * NT + threadIdx.x, GT = gridDim.x * NT;
+    const long long np = (long long)qn * BW;
+    for (long long t0 = (long long)gtid - (threadIdx.x & 31); t0 < np; t0 += GT) {  // warp-uniform trip count
+        const long long t = t0 + (threadIdx.x & 31);
+        double d = 0.0;
+        int u = -1;
+        if (t < np) {
+            u = __ldcg(&p.Q[qlo + (int)(t >> 6)]);
+            const int b = (int)(t & 63);
+            if ((__ldcg(&p.F[(size_t)u * p.LS + L]) >> b) & 1ull) {
+                const double su = __ldcg(p.sig + sidx(p, b, u));
+                if (su >= TWO53) c.inexact = 1;  // order-dependent sum of >= 3 terms possible
+                d = su * __ldcg(p.dacc + sidx(p, b, u));
+                if (p.dbg_delta) p.dbg_delta[(size_t)b * p.n + u] = d;
+            }
+        }
+        d = warp_sum(d);  // the 32 lanes share u (64 pairs per entry = 2 warps)
+        if ((threadIdx.x & 31) == 0 && u >= 0 && d != 0.0) atomicAdd(&p.bc[u], d);
+    }
+}
+
+__device__ __forceinline__ void trace_level(const BParams &p, int dir, int L, int A, long long t0, bool active) {
+    if ((threadIdx.x & 31) != 0 || !active) return;
+    long long *t = p.trace + ((size_t)dir * p.LS + L) * 12;
+    const long long dt = clock64() - t0;
+    atomicMax(&t[1], dt);
+    atomicAdd((unsigned long long *)&t[2], (unsigned long long)dt);
+    if (threadIdx.x == 0 && blockIdx.x == 0) t[3] = A;
+}
+
+// trace slots 4.. of a level: cycles in row windows, in pair lists, their counts, pairs,
+// cycles in the whole range
+__device__ __forceinline__ void trace_flush(const BParams &p, int dir, int L, long long *tp) {
+    if ((threadIdx.x & 31) != 0) return;
+    long long *t = p.trace + ((size_t)dir * p.LS + L) * 12 + 4;
+    for (int i = 0; i < 6; ++i)
+        if (tp[i]) atomicAdd((unsigned long long *)&t[i], (unsigned long long)tp[i]);
 }
 
 template <int NT>
-__global__ void __launch_bounds__(NT, 1024 / NT) batch_kernel(BParams p) {
+__global__ void __launch_bounds__(NT, 768 / NT) batch_kernel(BParams p) {
     if (p.sampled_flag && __ldcg(p.sampled_flag) == 0) return;  // Alg. 5 chose WE: bc_kernel runs
     cg::grid_group grid = cg::this_grid();
-    __shared__ int s_qlo[MAX_LCAP + 4];   // Q offset of each level
-    __shared__ int s_hlo[MAX_LCAP + 4];   // hub-entry offset of each level
-    __shared__ int s_hch[MAX_LCAP + 4];   // hub chunks of each level
-    __shared__ int s_ovf;
+    __shared__ int s_qlo[MAX_LCAP + 4];  // Q offset of each level
+    __shared__ int s_A[MAX_LCAP + 4];    // arcs of each level
+    __shared__ long long s_ovf;
+    __shared__ uint16_t s_lst[NT / 32][32 * BW];  // per-warp (arc, source) pair lists
+    uint16_t *lst = s_lst[threadIdx.x >> 5];
     const int lane = threadIdx.x & 31;
     const int gtid = blockIdx.x * NT + threadIdx.x, GT = gridDim.x * NT;
+    const int gw = gtid >> 5, GW = GT >> 5;
     const int LS = p.LS;
-    int *grab_f = p.grab, *hgrab_f = p.grab + LS, *grab_b = p.grab + 2 * LS, *hgrab_b = p.grab + 3 * LS;
-    Cnt c;
+    __shared__ unsigned long long s_cnt[NT / 32][4];  // per-warp totals over completed batches
+    __shared__ int s_inexact;
+    if (lane == 0)
+        for (int i = 0; i < 4; ++i) s_cnt[threadIdx.x >> 5][i] = 0ull;
+    if (threadIdx.x == 0) s_inexact = 0;
     const long long nbatch = (p.k + BW - 1) / BW;
 
     for (long long bt = 0; bt < nbatch; ++bt) {
         const long long b0 = bt * BW;
         const int nb = (int)min((long long)BW, p.k - b0);
         Cnt cb;  // this batch's counters, kept only if it completes (no overflow)
+        unsigned long long wor = 0ull;
         // ---- Alg. 1 for the batch: d_b(s_b) = 0, sigma_b(s_b) = 1
-        if (threadIdx.x == 0) {
-            s_qlo[0] = 0;
-            s_hlo[0] = 0;
-        }
+        if (threadIdx.x == 0) s_qlo[0] = 0;
         if (gtid < nb) {
             const int b = gtid;
             int s = p.sources ? p.sources[p.src_base + b0 + b] : (int)(p.src_base + b0 + b);
             if (p.perm) s = p.perm[s];
-            p.sig[(size_t)s * BW + b] = 1.0;
+            p.sig[sidx(p, b, s)] = 1.0;
             if (p.dbg_d) {
                 p.dbg_d[(size_t)b * p.n + s] = 0;
                 p.dbg_sigma[(size_t)b * p.n + s] = 1.0;
             }
-            if (atomicOr(&p.F[(size_t)s * LS], 1ull << b) == 0ull) {
-                p.Q[atomicAdd(&p.qcnt[0], 1)] = s;
-                const int deg = p.ro[s + 1] - p.ro[s];
-                if (deg > p.CH) hub_push(p, 0, 0, s, deg);
+            const int deg = p.ro[s + 1] - p.ro[s];
+            // isolated sources have no arcs: bit set, never expanded (every Q row has deg >= 1)
+            if (atomicOr(&p.F[(size_t)s * LS], 1ull << b) == 0ull && deg > 0) {
+                const unsigned long long old = atomicAdd(&p.qctr[0], CNT_ONE | (unsigned long long)deg);
+                p.Q[(int)(old >> 40)] = s;
+                p.qoff[(int)(old >> 40)] = (int)(old & ARC_MASK);
+            }
+            if (deg == 0) {  // its BFS is level 0 alone
+                cb.reached += 1;
+                atomicOr(&p.lvor[0], 1ull << b);
             }
         }
         grid.sync();
 
         // ---- forward (Alg. 2), one level per grid barrier
-        int L = 0, qlo = 0, hlo = 0;
+        Level lv;
+        lv.L = 0;
+        lv.qlo = 0;
         bool ovf = false;
         for (;;) {
-            const int qn = __ldcg(&p.qcnt[L]);
-            const unsigned long long hc = __ldcg(&p.hcnt[L]);
-            const int hn = (int)(hc >> 40), hch = (int)(hc & CH_MASK);
-            const int qlo_next = qlo + qn, hlo_next = hlo + hn;
+            const unsigned long long qc = __ldcg(&p.qctr[lv.L]);
+            lv.qn = (int)(qc >> 40);
+            lv.A = (int)(qc & ARC_MASK);
+            lv.qlo_next = lv.qlo + lv.qn;
+            lv.per = max(p.min_range, (lv.A + GW - 1) / GW);
             if (threadIdx.x == 0) {
-                s_qlo[L + 1] = qlo_next;
-                s_hlo[L + 1] = hlo_next;
-                s_hch[L] = hch;
+                s_qlo[lv.L + 1] = lv.qlo_next;
+                s_A[lv.L] = lv.A;
             }
-            unsigned long long wor = 0ull;
-            // hub chunks first (the long poles), then whole rows
-            for (;;) {
-                int ci = 0;
-                if (lane == 0) ci = atomicAdd(&hgrab_f[L], 1);
-                ci = __shfl_sync(FULL, ci, 0);
-                if (ci >= hch) break;
-                int pos = 0;
-                if (lane == 0) pos = hub_find(p, hlo, hn, ci);
-                pos = __shfl_sync(FULL, pos, 0);
-                const int h = __ldcg(&p.hv[pos]);
-                const int chunk = ci - __ldcg(&p.hb[pos]);
-                const int rb = __ldg(&p.ro[h]), re = __ldg(&p.ro[h + 1]);
-                const int a0 = rb + chunk * p.CH, a1 = min(re, a0 + p.CH);
-                const unsigned long long f = __ldcg(&p.F[(size_t)h * LS + L]);
-                double acc0 = 0.0, acc1 = 0.0;
-                if (L > 0) {
-                    fwd_seg<true>(p, L, f, a0, a1, qlo_next, hlo_next, acc0, acc1, cb);
-                    double *ha = p.hacc + (size_t)pos * BW;
-                    if (((f >> lane) & 1ull) && acc0 != 0.0) atomicAdd(ha + lane, acc0);
-                    if (((f >> (lane + 32)) & 1ull) && acc1 != 0.0) atomicAdd(ha + 32 + lane, acc1);
-                } else {
-                    fwd_seg<false>(p, L, f, a0, a1, qlo_next, hlo_next, acc0, acc1, cb);
-                }
-                if (lane == 0) {
-                    cb.sc += (unsigned long long)(a1 - a0);
-                    if (chunk == 0) {
-                        cb.reached += (unsigned long long)__popcll(f);
-                        cb.ar += (unsigned long long)__popcll(f) * (unsigned long long)(re - rb);
-                        wor |= f;
-                    }
-                }
+            const int nact = lv.A > 0 ? (lv.A + lv.per - 1) / lv.per : 0;
+            const long long t0 = clock64();
+            long long tp[6] = {0, 0, 0, 0, 0, 0};
+            long long *tpp = (p.trace && bt == 0) ? tp : nullptr;
+            if (gw < nact) process_range<true>(p, lv, gw * lv.per, min(lv.A, (gw + 1) * lv.per), cb, wor, lst, tpp);
+            if (tpp) trace_flush(p, 0, lv.L, tp);
+            if (p.trace && bt == 0) trace_level(p, 0, lv.L, lv.A, t0, gw < nact);
+            {
+                const unsigned lo32 = __reduce_or_sync(FULL, (unsigned)wor);
+                const unsigned hi32 = __reduce_or_sync(FULL, (unsigned)(wor >> 32));
+                const unsigned long long w64 = ((unsigned long long)hi32 << 32) | lo32;
+                if (lane == 0 && w64) atomicOr(&p.lvor[lv.L], w64);
             }
-            for (;;) {
-                int i0 = 0;
-                if (lane == 0) i0 = atomicAdd(&grab_f[L], GRAB);
-                i0 = __shfl_sync(FULL, i0, 0);
-                if (i0 >= qn) break;
-                const int cnt = min(GRAB, qn - i0);
-                int my_u = 0, my_b = 0, my_e = 0;
-                unsigned long long my_f = 0ull;
-                if (lane < cnt) {
-                    my_u = __ldcg(&p.Q[qlo + i0 + lane]);
-                    my_b = __ldg(&p.ro[my_u]);
-                    my_e = __ldg(&p.ro[my_u + 1]);
-                    my_f = __ldcg(&p.F[(size_t)my_u * LS + L]);
-                }
-                for (int j = 0; j < cnt; ++j) {
-                    const int u = __shfl_sync(FULL, my_u, j);
-                    const int rb = __shfl_sync(FULL, my_b, j), re = __shfl_sync(FULL, my_e, j);
-                    if (re - rb > p.CH) continue;  // hub: done by chunks
-                    const unsigned long long f = shfl64(my_f, j);
-                    double acc0 = 0.0, acc1 = 0.0;
-                    if (L > 0) {
-                        fwd_seg<true>(p, L, f, rb, re, qlo_next, hlo_next, acc0, acc1, cb);
-                        store_sigma(p, u, L, f, acc0, acc1);
-                    } else {
-                        fwd_seg<false>(p, L, f, rb, re, qlo_next, hlo_next, acc0, acc1, cb);
-                    }
-                    if (lane == 0) {
-                        cb.sc += (unsigned long long)(re - rb);
-                        cb.reached += (unsigned long long)__popcll(f);
-                        cb.ar += (unsigned long long)__popcll(f) * (unsigned long long)(re - rb);
-                        wor |= f;
-                    }
-                }
-            }
-            if (lane == 0 && wor) atomicOr(&p.lvor[L], wor);
+            wor = 0ull;
             grid.sync();
-            if (hn > 0 && L > 0) {  // hub sigma = sum of its chunks' partial pulls
-                for (int e = gtid >> 5; e < hn; e += GT >> 5) {
-                    const int pos = hlo + e;
-                    const int h = __ldcg(&p.hv[pos]);
-                    const unsigned long long f = __ldcg(&p.F[(size_t)h * LS + L]);
-                    double *ha = p.hacc + (size_t)pos * BW;
-                    const double v0 = __ldcg(ha + lane), v1 = __ldcg(ha + 32 + lane);
-                    ha[lane] = 0.0;
-                    ha[32 + lane] = 0.0;
-                    if ((((f >> lane) & 1ull) && v0 >= TWO53) || (((f >> (lane + 32)) & 1ull) && v1 >= TWO53))
-                        cb.inexact = 1;  // chunk partials were summed in arrival order
-                    store_sigma(p, h, L, f, v0, v1);
-                }
-                grid.sync();
+            if (p.trace && bt == 0 && gtid == 0) atomicAdd((unsigned long long *)&p.trace[lv.L * 12], (unsigned long long)(clock64() - t0));
+            const int qn1 = (int)(__ldcg(&p.qctr[lv.L + 1]) >> 40);
+            if (qn1 == 0) break;  // Q_next_len == 0 (Alg. 2 l.11)
+            if (lv.L + 1 > p.Lcap) {
+                ovf = true;
+                break;
             }
-            const int qn1 = __ldcg(&p.qcnt[L + 1]);
-            if (qn1 == 0) break;                    // Q_next_len == 0 (Alg. 2 l.11)
-            if (L + 1 > p.Lcap) { ovf = true; break; }
-            qlo = qlo_next;
-            hlo = hlo_next;
-            ++L;
+            lv.qlo = lv.qlo_next;
+            ++lv.L;
         }
-        const int Ltop = ovf ? L + 1 : L;  // deepest level holding Q entries
-        if (threadIdx.x == 0) {
-            const int qn1 = __ldcg(&p.qcnt[L + 1]);
-            const unsigned long long hc1 = __ldcg(&p.hcnt[L + 1]);
-            s_qlo[L + 2] = s_qlo[L + 1] + qn1;
-            s_hlo[L + 2] = s_hlo[L + 1] + (int)(hc1 >> 40);
-            s_ovf = 0;
-        }
+        const int Lmax = lv.L;
+        const int Ltop = ovf ? Lmax + 1 : Lmax;  // deepest level holding Q entries
+        if (threadIdx.x == 0) s_qlo[Lmax + 2] = s_qlo[Lmax + 1] + (int)(__ldcg(&p.qctr[Lmax + 1]) >> 40);
         __syncthreads();
 
-        // ---- backward (Alg. 3), deepest level first
         if (!ovf) {
-            for (int Lb = L; Lb >= 1; --Lb) {
-                const bool scan = Lb < L;  // the deepest level has no successors: delta = 0
-                const int bqlo = s_qlo[Lb], bqn = s_qlo[Lb + 1] - s_qlo[Lb];
-                const int bhlo = s_hlo[Lb], bhn = s_hlo[Lb + 1] - s_hlo[Lb], bhch = s_hch[Lb];
-                if (scan && bhn > 0) {
-                    for (;;) {
-                        int ci = 0;
-                        if (lane == 0) ci = atomicAdd(&hgrab_b[Lb], 1);
-                        ci = __shfl_sync(FULL, ci, 0);
-                        if (ci >= bhch) break;
-                        int pos = 0;
-                        if (lane == 0) pos = hub_find(p, bhlo, bhn, ci);
-                        pos = __shfl_sync(FULL, pos, 0);
-                        const int h = __ldcg(&p.hv[pos]);
-                        const int chunk = ci - __ldcg(&p.hb[pos]);
-                        const int rb = __ldg(&p.ro[h]), re = __ldg(&p.ro[h + 1]);
-                        const int a0 = rb + chunk * p.CH, a1 = min(re, a0 + p.CH);
-                        const unsigned long long f = __ldcg(&p.F[(size_t)h * LS + Lb]);
-                        double acc0 = 0.0, acc1 = 0.0;
-                        bwd_seg(p, Lb, f, a0, a1, acc0, acc1);
-                        double *ha = p.hacc + (size_t)pos * BW;
-                        if (((f >> lane) & 1ull) && acc0 != 0.0) atomicAdd(ha + lane, acc0);
-                        if (((f >> (lane + 32)) & 1ull) && acc1 != 0.0) atomicAdd(ha + 32 + lane, acc1);
-                        if (lane == 0) cb.sc += (unsigned long long)(a1 - a0);
-                    }
-                }
-                for (;;) {
-                    int i0 = 0;
-                    if (lane == 0) i0 = atomicAdd(&grab_b[Lb], GRAB);
-                    i0 = __shfl_sync(FULL, i0, 0);
-                    if (i0 >= bqn) break;
-                    const int cnt = min(GRAB, bqn - i0);
-                    int my_u = 0, my_b = 0, my_e = 0;
-                    unsigned long long my_f = 0ull;
-                    if (lane < cnt) {
-                        my_u = __ldcg(&p.Q[bqlo + i0 + lane]);
-                        my_b = __ldg(&p.ro[my_u]);
-                        my_e = __ldg(&p.ro[my_u + 1]);
-                        my_f = __ldcg(&p.F[(size_t)my_u * LS + Lb]);
-                    }
-                    for (int j = 0; j < cnt; ++j) {
-                        const int u = __shfl_sync(FULL, my_u, j);
-                        const int rb = __shfl_sync(FULL, my_b, j), re = __shfl_sync(FULL, my_e, j);
-                        if (scan && re - rb > p.CH) continue;  // hub: done by chunks
-                        const unsigned long long f = shfl64(my_f, j);
-                        double acc0 = 0.0, acc1 = 0.0;
-                        if (scan) {
-                            bwd_seg(p, Lb, f, rb, re, acc0, acc1);
-                            if (lane == 0) cb.sc += (unsigned long long)(re - rb);
-                        }
-                        const double bs = warp_sum(finish_pair(p, u, f, acc0, acc1));
-                        if (lane == 0 && bs != 0.0) atomicAdd(&p.bc[u], bs);
-                    }
-                }
+            // ---- backward (Alg. 3), deepest level first.  The deepest level's pairs have
+            // no successors: acc = 0 (zeroed at discovery), delta = 0, omega = 1 / sigma.
+            for (int Lb = Lmax - 1; Lb >= 1; --Lb) {
+                Level bl;
+                bl.L = Lb;
+                bl.qlo = s_qlo[Lb];
+                bl.qn = s_qlo[Lb + 1] - bl.qlo;
+                bl.A = s_A[Lb];
+                bl.qlo_next = s_qlo[Lb + 1];
+                bl.per = max(p.min_range, (bl.A + GW - 1) / GW);
+                const int nact = bl.A > 0 ? (bl.A + bl.per - 1) / bl.per : 0;
+                const long long t0 = clock64();
+                long long tp[6] = {0, 0, 0, 0, 0, 0};
+                long long *tpp = (p.trace && bt == 0) ? tp : nullptr;
+                if (gw < nact) process_range<false>(p, bl, gw * bl.per, min(bl.A, (gw + 1) * bl.per), cb, wor, lst, tpp);
+                if (tpp) trace_flush(p, 1, Lb, tp);
+                // level Lb + 1 is complete since the last barrier: its deltas into bc
+                if (Lb + 1 < Lmax) delta_pass<NT>(p, Lb + 1, s_qlo[Lb + 1], s_qlo[Lb + 2] - s_qlo[Lb + 1], cb);
+                if (p.trace && bt == 0) trace_level(p, 1, Lb, bl.A, t0, gw < nact);
                 grid.sync();
-                if (scan && bhn > 0) {
-                    for (int e = gtid >> 5; e < bhn; e += GT >> 5) {
-                        const int pos = bhlo + e;
-                        const int h = __ldcg(&p.hv[pos]);
-                        const unsigned long long f = __ldcg(&p.F[(size_t)h * LS + Lb]);
-                        double *ha = p.hacc + (size_t)pos * BW;
-                        const double v0 = __ldcg(ha + lane), v1 = __ldcg(ha + 32 + lane);
-                        ha[lane] = 0.0;
-                        ha[32 + lane] = 0.0;
-                        const double bs = warp_sum(finish_pair(p, h, f, v0, v1));
-                        if (lane == 0 && bs != 0.0) atomicAdd(&p.bc[h], bs);
+                if (p.trace && bt == 0 && gtid == 0) atomicAdd((unsigned long long *)&p.trace[((LS + Lb) * 12)], (unsigned long long)(clock64() - t0));
+            }
+            if (Lmax >= 2) delta_pass<NT>(p, 1, s_qlo[1], s_qlo[2] - s_qlo[1], cb);
+            if (p.dbg_d) {  // debug export: d and sigma of every pair
+                for (int l = 1; l <= Lmax; ++l) {
+                    const long long np = (long long)(s_qlo[l + 1] - s_qlo[l]) * BW;
+                    for (long long t = gtid; t < np; t += GT) {
+                        const int u = __ldcg(&p.Q[s_qlo[l] + (int)(t >> 6)]);
+                        const int b = (int)(t & 63);
+                        if ((__ldcg(&p.F[(size_t)u * LS + l]) >> b) & 1ull) {
+                            p.dbg_d[(size_t)b * p.n + u] = l;
+                            p.dbg_sigma[(size_t)b * p.n + u] = __ldcg(p.sig + sidx(p, b, u));
+                        }
                     }
-                    grid.sync();
                 }
             }
+            grid.sync();
         } else if (blockIdx.x == 0) {
             // more than Lcap + 1 levels: this batch's sources go to the per-source kernel
-            if (threadIdx.x == 0) s_ovf = (int)atomicAdd((unsigned long long *)p.ovf_n, (unsigned long long)nb);
+            if (threadIdx.x == 0) s_ovf = (long long)atomicAdd((unsigned long long *)p.ovf_n, (unsigned long long)nb);
             __syncthreads();
             for (int b = threadIdx.x; b < nb; b += NT)
                 p.ovf_src[s_ovf + b] = p.sources ? p.sources[p.src_base + b0 + b] : (int)(p.src_base + b0 + b);
         }
 
-        // ---- reset for the next batch: masks of every Q entry, level counters
-        for (int l = 0; l <= Ltop; ++l)
+        // ---- reset for the next batch: masks of every Q entry and of the sources, counters
+        for (int l = 1; l <= Ltop; ++l)
             for (int i = s_qlo[l] + gtid; i < s_qlo[l + 1]; i += GT) p.F[(size_t)__ldcg(&p.Q[i]) * LS + l] = 0ull;
+        if (gtid < nb) {
+            int s = p.sources ? p.sources[p.src_base + b0 + gtid] : (int)(p.src_base + b0 + gtid);
+            if (p.perm) s = p.perm[s];
+            p.F[(size_t)s * LS] = 0ull;
+        }
         if (blockIdx.x == 0) {
-            for (int l = threadIdx.x; l <= Ltop + 1 && l < LS; l += NT) {
-                p.qcnt[l] = 0;
-                p.hcnt[l] = 0ull;
-                grab_f[l] = hgrab_f[l] = grab_b[l] = hgrab_b[l] = 0;
-            }
+            for (int l = threadIdx.x; l <= Ltop + 1 && l < LS; l += NT) p.qctr[l] = 0ull;
             if (threadIdx.x < 32) {
-                unsigned long long lv = 0;
+                unsigned long long lvs = 0;
                 for (int l = threadIdx.x; l <= Ltop && l < LS; l += 32) {
-                    lv += (unsigned long long)__popcll(__ldcg(&p.lvor[l]));
+                    lvs += (unsigned long long)__popcll(__ldcg(&p.lvor[l]));
                     p.lvor[l] = 0ull;
                 }
 #pragma unroll
-                for (int o = 16; o > 0; o >>= 1) lv += __shfl_xor_sync(FULL, lv, o);
+                for (int o = 16; o > 0; o >>= 1) lvs += __shfl_xor_sync(FULL, lvs, o);
                 if (threadIdx.x == 0) {
                     if (!ovf) {
-                        atomicAdd(&p.stats->levels, lv);
-                        atomicAdd(&p.stats->we_levels, lv);
+                        atomicAdd(&p.stats->levels, lvs);
+                        atomicAdd(&p.stats->we_levels, lvs);
                         atomicAdd(&p.stats->sources, (unsigned long long)nb);
                     } else {
                         atomicAdd(&p.stats->batch_overflows, 1ull);
@@ -444,40 +540,33 @@ __global__ void __launch_bounds__(NT, 1024 / NT) batch_kernel(BParams p) {
                 }
             }
         }
-        if (!ovf) {
-            c.reached += cb.reached;
-            c.ar += cb.ar;
-            c.dag += cb.dag;
-            c.sc += cb.sc;
+        if (!ovf) {  // overflowed batches are counted by the per-source rerun
+            unsigned long long v[4] = {cb.reached, cb.ar, cb.dag, cb.sc};
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) v[i] += __shfl_xor_sync(FULL, v[i], o);
+                if (lane == 0) s_cnt[threadIdx.x >> 5][i] += v[i];
+            }
         }
-        c.inexact |= cb.inexact;
+        if (cb.inexact) s_inexact = 1;
         grid.sync();
     }
 
-    // per-warp flush of the byte-model counters; overflowed batches are
-    // counted by the per-source kernel that reruns them
-    unsigned long long r = c.reached, a = c.ar, d = c.dag, s = c.sc;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        r += __shfl_xor_sync(FULL, r, o);
-        a += __shfl_xor_sync(FULL, a, o);
-        d += __shfl_xor_sync(FULL, d, o);
-        s += __shfl_xor_sync(FULL, s, o);
-    }
-    const int inex = __any_sync(FULL, c.inexact);
+    // per-warp flush of the byte-model counters
+    __syncthreads();
     if (lane == 0) {
-        if (r) atomicAdd(&p.stats->n_reached, r);
-        if (a) atomicAdd(&p.stats->arcs_reached, a);
-        if (d) atomicAdd(&p.stats->dag_arcs, d);
-        if (s) atomicAdd(&p.stats->arcs_scanned, s);
-        if (inex) atomicOr(&p.stats->sigma_inexact, 1);
+        const unsigned long long *v = s_cnt[threadIdx.x >> 5];
+        if (v[0]) atomicAdd(&p.stats->n_reached, v[0]);
+        if (v[1]) atomicAdd(&p.stats->arcs_reached, v[1]);
+        if (v[2]) atomicAdd(&p.stats->dag_arcs, v[2]);
+        if (v[3]) atomicAdd(&p.stats->arcs_scanned, v[3]);
     }
+    if (threadIdx.x == 0 && s_inexact) atomicOr(&p.stats->sigma_inexact, 1);
 }
 
 const void *batch_kernel_fn(int nt) {
-    return nt == 128 ? (const void *)batch_kernel<128>
-           : nt == 512 ? (const void *)batch_kernel<512>
-                       : (const void *)batch_kernel<256>;
+    return nt == 128 ? (const void *)batch_kernel<128> : (const void *)batch_kernel<256>;
 }
 
 }  // namespace bcbatch

@@ -5,10 +5,9 @@
 // delta of every source are unchanged), scheduled differently: source b of a batch owns
 // bit b of a 64-bit mask per vertex and level, F_L[v] = { b : d_b(v) = L }.  A vertex v
 // is expanded once per level L at which ANY source of the batch has it (the union of the
-// 64 frontiers), so each CSR row read serves every source that has v at that level
-// (Kepler-era design expanded it once per source).  Warp lanes map to
-// sources (lane l owns sources l and l+32), so the sigma / omega gathers of one arc are
-// one coalesced 512-byte row of a vertex-major [n][64] fp64 array.
+// 64 frontiers, Q_L), so each CSR row read serves every source that has v at that level
+// (the Kepler design expanded it once per source).  Warp lanes map to
+// sources only inside rows long enough to fill a window (hubs); elsewhere lanes = pairs.
 //
 //   forward level L, u in Q_L, f = F_L[u], for x in N(u) (CSR order):
 //     sigma pull (Alg. 2 l.7-8 as a pull, R18): b in f & F_{L-1}[x] -> acc_b += sigma_b(x)
@@ -19,8 +18,15 @@
 //     delta_b(u) = sigma_b(u) * acc_b, omega_b(u) = (1 + delta_b(u)) / sigma_b(u),
 //     bc[u] += sum_b delta_b(u)  (Eq. 3)
 //
-// Rows longer than CH arcs ("hubs") are split into CH-arc chunks spread over the grid;
-// their partial sums meet in hacc and are finished after one more grid barrier.
+// Arc-parallel accumulation: each level's rows form one arc space [0, A_L) (Q entries
+// carry their arc offset, assigned with the entry by one packed 64-bit atomic at enqueue
+// time), cut into equal contiguous ranges, one per warp, lanes = arcs whatever the row
+// boundaries.  Every (arc, source) pair of the DAG is one lane-parallel gather plus one
+// fire-and-forget fp64 reduction into the row's accumulator:
+//   forward  sigma_b(u) += sigma_b(x)                 (sigma_b(u) zeroed when (u, b) is discovered)
+//   backward acc_b(u)   += 1/sigma_b(x) + acc_b(x)    (= omega_b(x) = (1 + delta_b(x)) / sigma_b(x))
+// and delta_b(u) = sigma_b(u) * acc_b(u) is added to bc[u] one level later.  Sums of
+// integers below 2^53 are exact in any order, so sigma stays bit-exact there.
 #pragma once
 
 #include <cstdint>
@@ -44,29 +50,31 @@ struct BParams {
     long long src_base, k;        // this launch's sources: [src_base, src_base + k) of the list
     int Lcap;                     // levels 0..Lcap can be expanded; deeper => overflow
     int LS;                       // Lcap + 2: mask words per vertex (vertex-major F)
-    int CH;                       // hub chunk length (arcs); rows with deg > CH are split
+    int min_range;                // minimum arcs per warp range
     unsigned long long *F;        // F[v * LS + L] (zero between batches)
-    double *sig;                  // sig[v * 64 + b]: sigma_b(v), then omega_b(v) in place
+    size_t sn;                    // n rounded up to 32 (allocation)
+    double *sig;                  // sig[v * 64 + b]: sigma_b(v)
+    double *dacc;                 // dacc[v * 64 + b]: sum of omega_b over v's successors
     int *Q;                       // union frontiers, level after level; capacity qcap
+    int *qoff;                    // arc offset of each Q entry within its level
     long long qcap;
-    int *qcnt;                    // [LS] entries per level
-    unsigned long long *hcnt;     // [LS] hub entries per level, packed (count << 40 | chunks)
-    int *grab, *hgrab;            // [LS] work counters (vertices / hub chunks)
+    unsigned long long *qctr;     // [LS] per level, packed (entries << 40 | arcs)
     unsigned long long *lvor;     // [LS] OR of the level's masks (levels statistic)
-    int *hv, *hb;                 // hub entries: vertex, first chunk index within its level
-    double *hacc;                 // [hcap][64] hub partial sums (zero between uses)
-    long long hcap;
     double *bc;                   // BC in internal ids (accumulated with atomics)
     bcdev::DevStats *stats;
     const int *sampled_flag;      // non-NULL: run only if *sampled_flag == 1 (Alg. 5 EP run)
     int *ovf_src;                 // sources of batches that exceeded Lcap (caller ids)
     long long *ovf_n;
+    // per-level trace of batch 0 (tools/batch_trace.py), may be NULL:
+    // trace[((dir * LS) + L) * 4 + {0 wall cycles (CTA 0), 1 max warp busy cycles,
+    //                               2 sum warp busy cycles, 3 arcs}], dir 0 fwd / 1 bwd
+    long long *trace;
     // debug export of one launch (<= 64 sources), internal ids, [64][n]; may be NULL
     int *dbg_d;
     double *dbg_sigma, *dbg_delta;
 };
 
-// Kernel symbol for a block size (128, 256 or 512 threads); launched cooperatively.
+// Kernel symbol for a block size (128 or 256 threads); launched cooperatively.
 const void *batch_kernel_fn(int nt);
 
 }  // namespace bcbatch

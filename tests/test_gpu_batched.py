@@ -4,9 +4,9 @@ against the CPU oracle, through the C ABI.
 Same bar as tests/test_gpu_parity.py: d bit-exact; sigma bit-exact wherever the
 oracle's sigma is below 2^53 (rows are pulled in CSR order, the oracle's order), within
 1e-12 relative above; delta and BC within 1e-9 (|gpu - ref| / max(|ref|, 1)).
-Batches of 64 sources: full batches, ragged tails (k mod 64 != 0), duplicates, hub
-rows split into chunks (hub_chunk small), batches deeper than the level cap (rerun
-per source), and the auto engine choosing batched only for Alg. 5 EP runs.
+Batches of 64 sources: full batches, ragged tails (k mod 64 != 0), duplicates, rows
+split across many warp ranges (hub_chunk small), batches deeper than the level cap
+(rerun per source), and the auto engine's choice (Alg. 5 EP run on a large skewed graph).
 """
 import numpy as np
 import pytest
@@ -108,7 +108,8 @@ def test_c1_batched_stats_match_oracle_counters(bcmod, oracle_mod):
 
 @pytest.mark.parametrize("chunk", [4, 33, 200])
 def test_c1_hub_chunks(bcmod, oracle_mod, chunk):
-    """Rows longer than hub_chunk are split over warps (partial sums meet in hacc)."""
+    """hub_chunk = minimum arcs per warp range: tiny ranges split every row over many
+    warps, whose fp64 reductions meet in the row's accumulators."""
     g = graph("c1")
     with bcmod.BCGraph.from_graph(g, engine="batched", strategy="we", hub_chunk=chunk) as bg:
         check_bc(bg, g, None, oracle_mod)
@@ -167,14 +168,21 @@ def test_delaunay_batched_sigma_above_2p53(bcmod, oracle_mod):
 
 
 def test_auto_engine_follows_alg5(bcmod, oracle_mod):
-    """Auto: a SAMPLING run whose Alg. 5 decision is EP (small-world) runs batched."""
-    g = graph("c4")
-    src = gg.sample_sources(g, 512 + 200, seed=9)
+    """Auto: batched only for an Alg. 5 EP run on a large skewed graph (c5k); c4 and the
+    high-diameter lattice stay per source."""
+    g = graph("c5k")
+    src = gg.sample_sources(g, 512 + 128, seed=9)
     with bcmod.BCGraph.from_graph(g) as bg:  # defaults: sampling, auto engine
         check_bc(bg, g, src, oracle_mod, nthreads=16)
         st = bg.stats()
-        assert st["sampling_ep"] == 1 and st["batches"] == (200 + 63) // 64
+        assert st["sampling_ep"] == 1 and st["batches"] == 2
         assert st["sources"] == src.size
+    g4 = graph("c4")
+    src4 = gg.sample_sources(g4, 512 + 64, seed=9)
+    with bcmod.BCGraph.from_graph(g4) as bg:
+        check_bc(bg, g4, src4, oracle_mod, nthreads=16)
+        st = bg.stats()
+        assert st["sampling_ep"] == 1 and st["batches"] == 0
     g2 = gg.lattice2d(64, 64)  # high diameter: Alg. 5 -> WE -> per-source engine
     with bcmod.BCGraph.from_graph(g2) as bg:
         src2 = np.arange(0, g2.n, 7, dtype=np.int32)
