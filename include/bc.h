@@ -89,12 +89,12 @@ typedef struct bc_options {
     /* Implementation knobs (do not change results beyond fp64 rounding order): */
     int32_t block_threads;   /* threads per CTA: 0 = auto, 128, 256, 512 or 1024                */
     int32_t seq_max_deg;     /* rows up to this degree are summed by one thread in CSR order;
-                                longer rows CTA-cooperatively.  0 = auto (32)                  */
+                                longer rows cooperatively.  0 = auto (128)                     */
     int32_t level_store;     /* 0 = auto, 1 = exact int32 d in HBM, 2 = 2-bit codes in shared
                                 memory (undirected graphs whose codes fit; else EINVAL),
                                 3 = 2-bit codes in HBM/L2 (undirected graphs)                  */
     int32_t warp_max_deg;    /* rows up to this degree are expanded by one warp, longer rows
-                                by the whole CTA.  0 = auto (4096)                             */
+                                by the whole CTA.  0 = auto (16384)                            */
     int32_t l2_persist;      /* 0 = auto (on), -1 = off: persisting-L2 access-policy window
                                 over the CSR arrays during traversal launches                  */
     int32_t sort_frontier;   /* 0 = auto, 1 = on, -1 = off: rebuild large BFS levels in vertex

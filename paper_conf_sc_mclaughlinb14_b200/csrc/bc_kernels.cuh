@@ -390,7 +390,7 @@ __device__ __forceinline__ double coop_sum(const int *__restrict__ cols, int b, 
 // (also in mode 2, which skips non-successor slots: they only ever added 0.0).
 // cols must be 16-byte aligned with >= 3 ints of readable slack after the end.
 template <class Probe, class Gather, class Claim, class Visit>
-__device__ __forceinline__ double seq_row(const int *__restrict__ cols, int a, int e, const ArcBits &ab,
+__device__ __forceinline__ double seq_row_bits(const int *__restrict__ cols, int a, int e, const ArcBits &ab,
                                           Probe &probe, Gather &gather, Claim &claim, Visit &visit) {
     double acc = 0.0;
     // Successor bits of the row through a 64-arc window of two bitmap words starting at
@@ -463,6 +463,47 @@ __device__ __forceinline__ double seq_row(const int *__restrict__ cols, int a, i
     if (ab.mode == 1) {
         if ((uint32_t)win) atomicOr(&ab.sb[w0], (uint32_t)win);
         if (win >> 32) atomicOr(&ab.sb[w0 + 1], (uint32_t)(win >> 32));
+    }
+    return acc;
+}
+
+// Mode-0 row (no successor bitmap), software-pipelined: the column quad of step i+1 is
+// loaded while the probes / gathers / discoveries of step i are in flight.  Same slot
+// order and +0.0 padding as seq_row_bits, so the sum is unchanged.
+template <class Probe, class Gather, class Claim, class Visit>
+__device__ __forceinline__ double seq_row(const int *__restrict__ cols, int a, int e, const ArcBits &ab,
+                                          Probe &probe, Gather &gather, Claim &claim, Visit &visit) {
+    if (ab.mode != 0) return seq_row_bits(cols, a, e, ab, probe, gather, claim, visit);
+    double acc = 0.0;
+    int q = a & ~3;
+    if (q >= e) return acc;
+    int4 nx = *reinterpret_cast<const int4 *>(cols + q);
+    for (; q < e; q += 4) {
+        const int4 c4 = nx;
+        if (q + 4 < e) nx = *reinterpret_cast<const int4 *>(cols + q + 4);
+        unsigned valid = 0xFu;
+        if (q < a) valid &= 0xFu << (a - q);
+        if (q + 4 > e) valid &= 0xFu >> (q + 4 - e);
+        int u[4] = {c4.x, c4.y, c4.z, c4.w}, k[4];
+        bool ok[4];
+        double g[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            ok[j] = (valid >> j) & 1u;
+            u[j] = ok[j] ? u[j] : 0;
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) k[j] = probe(u[j]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) g[j] = ok[j] ? gather(u[j], k[j]) : 0.0;
+        bool won[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) won[j] = ok[j] && claim(u[j], k[j]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+            if (ok[j]) visit(u[j], k[j], won[j]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc += g[j];
     }
     return acc;
 }

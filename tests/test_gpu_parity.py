@@ -425,3 +425,17 @@ def test_extrapolate_and_normalize(bcmod, oracle_mod, flags):
     with bcmod.BCGraph.from_graph(g, extrapolate=extrapolate, normalize=normalize) as bg:
         got = bg.compute(src)
     assert np.max(np.abs(got - ref) / np.maximum(np.abs(ref), 1e-300)) < 1e-9
+
+
+@pytest.mark.parametrize("seq,warp", [(4, 8), (8, 200), (32, 4096), (128, 16384), (1024, 1024)])
+def test_row_split_knobs(bcmod, oracle_mod, seq, warp):
+    """Rows summed by one thread (deg <= seq), one warp (<= warp) or the whole CTA:
+    every split gives identical d/sigma (integers < 2^53) and BC within tolerance."""
+    for key, k in (("c1", None), ("c4", 120)):
+        g = graph(key)
+        src = None if k is None else gg.CONFIGS[key].sources(g)[:k]
+        with bcmod.BCGraph.from_graph(g, strategy="we", seq_max_deg=seq, warp_max_deg=warp) as bg:
+            check_bc(bg, g, src, oracle_mod)
+            hub = int(np.argmax(g.degrees()))
+            check_source(bg, g, hub, oracle_mod)
+            check_source(bg, g, 3 if src is None else int(src[0]), oracle_mod)
