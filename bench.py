@@ -61,11 +61,14 @@ def peaks():
 # ---------------------------------------------------------------- workload
 
 
-def make_workload(cfg_key: str, world: int, rank: int, scaling: str):
+def make_workload(cfg_key: str, world: int, rank: int, scaling: str, k_override: int = 0):
     from paper_conf_sc_mclaughlinb14_b200 import graphgen as gg
     from paper_conf_sc_mclaughlinb14_b200.distributed import shard_sources
     cfg = gg.CONFIGS[cfg_key]
     g = cfg.graph()
+    if k_override:                        # --sources: a bounded prefix of the workload
+        import dataclasses
+        cfg = dataclasses.replace(cfg, k=k_override)
     if cfg.k is None:                     # exact BC: all vertices
         total = np.arange(g.n, dtype=np.int32)
         local = shard_sources(total, rank, world, seed=cfg.seed)
@@ -166,7 +169,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
-    cfg, g, total, _ = make_workload(args.config, world, 0, args.scaling)
+    cfg, g, total, _ = make_workload(args.config, world, 0, args.scaling, args.sources)
     cores = len(os.sched_getaffinity(0))
     per_step = max(5.0, 150.0 / max(1, args.steps + args.warmup))
     import oracle
@@ -213,7 +216,8 @@ def bench_options(args):
 
 
 def workload_config(cfg, g, total, world, args):
-    return {"workload": f"{cfg.key}: {cfg.description}", "graph": g.name, "n": g.n, "m": g.m,
+    desc = cfg.description + (f" (bounded: --sources {args.sources} per GPU)" if args.sources else "")
+    return {"workload": f"{cfg.key}: {desc}", "graph": g.name, "n": g.n, "m": g.m,
             "sources_total": int(total.size), "sources_per_gpu": int(math.ceil(total.size / world)),
             "strategy": args.strategy, "options": bench_options(args),
             "parallelism": f"sources split over {world} GPU(s)",
@@ -236,7 +240,7 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=dev)
 
     t0 = time.time()
-    cfg, g, total, local = make_workload(args.config, world, rank, args.scaling)
+    cfg, g, total, local = make_workload(args.config, world, rank, args.scaling, args.sources)
     log(f"rank {rank}: graph {g.name} n={g.n} m={g.m} local sources {local.size} "
         f"(gen {time.time() - t0:.1f}s)")
     bg = bcm.BCGraph.from_graph(g, device=local_rank, **bench_options(args))
@@ -384,8 +388,10 @@ def main():
     ap.add_argument("--paper-params", action="store_true",
                     help="use the paper's EP guard (512) instead of the B200-retuned one")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
-    ap.add_argument("--engine", default="auto", choices=["auto", "per_source", "batched"],
+    ap.add_argument("--engine", default="auto", choices=["auto", "per_source", "batched", "group"],
                     help="source scheduling (include/bc.h BC_ENGINE_*)")
+    ap.add_argument("--sources", type=int, default=0,
+                    help="sources per GPU (0 = the config's own count); bounds c5 runs")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()

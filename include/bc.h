@@ -68,10 +68,16 @@ enum {
                                  there only)                                   */
     BC_ENGINE_PER_SOURCE = 1, /* one CTA per source (bc_kernel), every level WE or EP as the
                                  strategy chooses                                            */
-    BC_ENGINE_BATCHED = 2     /* undirected graphs: 64 sources per batch, level-synchronous
+    BC_ENGINE_BATCHED = 2,    /* undirected graphs: 64 sources per batch, level-synchronous
                                  over the whole GPU, one 64-bit source mask per vertex and
                                  level; every union-frontier row is read once per level for
                                  all 64 sources (work-efficient, queue-driven expansion)    */
+    BC_ENGINE_GROUP = 3       /* undirected graphs, work-efficient levels only (WE strategy,
+                                 or SAMPLING with an EP guard above n): the CTAs are split
+                                 into groups, each group traverses ONE source at a time with
+                                 a group barrier per level, so only a few sources' state is
+                                 live (L2-resident on large graphs); other launches fall back
+                                 to the per-source engine                                   */
 };
 
 typedef struct bc_graph bc_graph; /* opaque; owns device copies of the graph and workspace */
@@ -114,6 +120,8 @@ typedef struct bc_options {
     int32_t hub_chunk;       /* batched engine: minimum arcs per warp range when a BFS level's
                                 arcs are cut into equal warp ranges (rows of any length are
                                 split across ranges); 0 = auto 64                            */
+    int32_t group_ctas;      /* group engine: CTAs per group; 0 = auto (as many groups as keep
+                                their sigma + level codes + bitmaps within ~48 MB of L2)     */
 } bc_options;
 
 typedef struct bc_stats {

@@ -19,8 +19,8 @@ LIB_PATH = os.path.join(_HERE, "libbc.so")
 BC_OK, BC_EINVAL, BC_ENOMEM, BC_ECUDA, BC_EINTERNAL = 0, -1, -2, -3, -4
 BC_STRATEGY_WE, BC_STRATEGY_EP, BC_STRATEGY_HYBRID, BC_STRATEGY_SAMPLING = 0, 1, 2, 3
 STRATEGIES = {"we": 0, "ep": 1, "hybrid": 2, "sampling": 3}
-BC_ENGINE_AUTO, BC_ENGINE_PER_SOURCE, BC_ENGINE_BATCHED = 0, 1, 2
-ENGINES = {"auto": 0, "per_source": 1, "batched": 2}
+BC_ENGINE_AUTO, BC_ENGINE_PER_SOURCE, BC_ENGINE_BATCHED, BC_ENGINE_GROUP = 0, 1, 2, 3
+ENGINES = {"auto": 0, "per_source": 1, "batched": 2, "group": 3}
 BATCH_WIDTH = 64  # sources per batch of the batched engine
 
 EXPORTED = ("bc_graph_create", "bc_compute", "bc_compute_device", "bc_single_source",
@@ -38,7 +38,7 @@ class bc_options(ctypes.Structure):
                 ("sort_frontier", ctypes.c_int32), ("extrapolate", ctypes.c_int32),
                 ("normalize", ctypes.c_int32), ("succ_bits", ctypes.c_int32),
                 ("engine", ctypes.c_int32), ("batch_levels", ctypes.c_int32),
-                ("hub_chunk", ctypes.c_int32)]
+                ("hub_chunk", ctypes.c_int32), ("group_ctas", ctypes.c_int32)]
 
 
 class bc_stats(ctypes.Structure):

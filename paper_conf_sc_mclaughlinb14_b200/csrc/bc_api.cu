@@ -7,6 +7,7 @@
 #include "bc.h"
 #include "bc_kernels.cuh"
 #include "bc_batch.cuh"
+#include "bc_group.cuh"
 
 #include <algorithm>
 #include <cmath>
@@ -125,6 +126,14 @@ struct bc_graph {
         long long *ovf_n = nullptr;
     } bt;
     int batch_ran = 0;       // the last compute call launched the batched engine
+    // group engine (bc_group.cu); allocated on first use
+    struct Group {
+        int ready = 0, nt = 512, grid = 0, G = 0, code_words = 0, sb = 0;
+        unsigned long long *ctl = nullptr;
+        double *sigma = nullptr;
+        int *S = nullptr, *ends = nullptr, *bigq = nullptr;
+        uint32_t *codes = nullptr, *nb = nullptr, *sbits = nullptr;
+    } gr;
 };
 
 extern "C" void bc_default_options(bc_options *o) {
@@ -378,11 +387,151 @@ static int alloc_batch(bc_graph *g, long long max_sources) {
 // is far beyond L2 AND the degree distribution is skewed (relabelled graphs: c5k
 // 1.26x), loses on c4 (n = 2^18), on the unskewed small world c5ws and on every
 // high-diameter graph; the device-side Alg. 5 flag still has to say EP.
+static bool main_on_group(const bc_graph *g);
+
 static bool batch_wanted(const bc_graph *g) {
     if (g->directed || g->n == 0) return false;
     if (g->opt.engine == BC_ENGINE_BATCHED) return true;
     return g->opt.engine == BC_ENGINE_AUTO && g->opt.strategy == BC_STRATEGY_SAMPLING &&
-           g->perm != nullptr && g->n >= (1 << 21);
+           g->perm != nullptr && g->n >= (1 << 21) && !main_on_group(g);
+}
+
+static void free_group(bc_graph *g) {
+    bc_graph::Group &q = g->gr;
+    cudaFree(q.ctl);
+    cudaFree(q.sigma);
+    cudaFree(q.S);
+    cudaFree(q.ends);
+    cudaFree(q.bigq);
+    cudaFree(q.codes);
+    cudaFree(q.nb);
+    cudaFree(q.sbits);
+    q = bc_graph::Group{};
+}
+
+// Groups for the group engine: as many as keep every group's per-source state
+// (sigma 8n + codes n/4 + bitmaps 3n/8 + successor bits 2m/8 bytes) within ~48 MB of L2
+// together, at least one; group_ctas > 0 fixes the CTAs per group instead.
+static int group_count(const bc_graph *g, int grid) {
+    if (g->opt.group_ctas > 0) return std::max(1, std::min(grid, grid / g->opt.group_ctas));
+    // Auto, from the B200 sweep (kernel ms for 2,048 sources): the unskewed
+    // small world c5ws is fastest with 4 groups of 74 CTAs (1604 ms; 1 group 1918, 8 groups
+    // 1667), the skewed Kronecker c5k with groups of 9 CTAs (2479 ms; 18: 2873, 37: 3761,
+    // 4: 2505).  Skewed = internally relabelled by degree (want_reorder).
+    const int ctas = g->perm ? 9 : std::max(1, grid / 4);
+    return std::max(1, std::min(grid, grid / ctas));
+}
+
+static int alloc_group(bc_graph *g) {
+    bc_graph::Group &q = g->gr;
+    const int nt = g->n >= (1 << 17) ? 512 : 256;
+    int per_sm = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bcgroup::group_kernel_fn(nt), nt, 0));
+    if (per_sm < 1) return fail(BC_EINTERNAL, "group kernel cannot be resident");
+    const int grid = per_sm * g->num_sms;
+    const int G = group_count(g, grid);
+    const int sbw = g->opt.succ_bits >= 0;  // on unless switched off
+    if (q.ready && q.nt == nt && q.grid == grid && q.G == G && q.sb == sbw) return BC_OK;
+    free_group(g);
+    q.nt = nt;
+    q.grid = grid;
+    q.G = G;
+    q.sb = sbw;
+    q.code_words = (int)((((size_t)g->n + 63) / 64) * 4);
+    const size_t ng = (size_t)G;
+    CK(cudaMalloc(&q.ctl, ng * bcgroup::CTL_WORDS * 8));
+    CK(cudaMalloc(&q.sigma, ng * g->stride_n * sizeof(double)));
+    CK(cudaMalloc(&q.S, ng * g->stride_n * sizeof(int)));
+    CK(cudaMalloc(&q.ends, ng * g->stride_e * sizeof(int)));
+    CK(cudaMalloc(&q.bigq, (size_t)grid * g->stride_big * sizeof(int)));
+    CK(cudaMalloc(&q.codes, ng * (size_t)q.code_words * 4));
+    CK(cudaMalloc(&q.nb, ng * 3 * (size_t)g->nb_words * 4));
+    CK(cudaMemset(q.codes, 0, ng * (size_t)q.code_words * 4));
+    CK(cudaMemset(q.nb, 0, ng * 3 * (size_t)g->nb_words * 4));
+    if (sbw) {
+        CK(cudaMalloc(&q.sbits, ng * (size_t)g->sb_words * 4));
+        CK(cudaMemset(q.sbits, 0, ng * (size_t)g->sb_words * 4));
+    }
+    CK(cudaMemset(q.sigma, 0, ng * g->stride_n * sizeof(double)));
+    CK(cudaDeviceSynchronize());
+    q.ready = 1;
+    return BC_OK;
+}
+
+// Whether a launch may run on the group engine: undirected, every level work-efficient
+// (WE strategy, or Alg. 5 with a guard no frontier can reach), no device-side count.
+static bool group_eligible(const bc_graph *g, const KParams &p) {
+    if (g->directed || g->n == 0 || p.k_dev || p.skip_if_ep) return false;
+    return p.launch_mode == LM_WE ||
+           (p.launch_mode == LM_SAMPLED && (long long)p.ep_min_frontier > (long long)g->n);
+}
+
+// Auto mode picks the group engine for large undirected graphs (n >= 2^21: the c5
+// configs, where it beats the per-source engine 1.55x (c5ws) and 1.36x (c5k) and the
+// batched engine 2.2x / 1.14x); on smaller graphs the per-source engine
+// (codes in shared memory, ~300 sources in flight) is faster (c4: 728 vs 1374 ms).
+static bool group_auto(const bc_graph *g) {
+    return g->opt.engine == BC_ENGINE_AUTO && !g->directed && g->n >= (1 << 21);
+}
+
+static bool group_wanted(const bc_graph *g, const KParams &p) {
+    return (g->opt.engine == BC_ENGINE_GROUP || group_auto(g)) && group_eligible(g, p);
+}
+
+// Whether the main phase of a compute call runs entirely on the group engine.
+static bool main_on_group(const bc_graph *g) {
+    const int st = g->opt.strategy;
+    const bool all_we = st == BC_STRATEGY_WE ||
+                        (st == BC_STRATEGY_SAMPLING && (long long)g->opt.ep_min_frontier > (long long)g->n);
+    return (g->opt.engine == BC_ENGINE_GROUP || group_auto(g)) && !g->directed && g->n > 0 && all_we;
+}
+
+static int launch_group(bc_graph *g, const KParams &p0, cudaStream_t st) {
+    int rc = alloc_group(g);
+    if (rc) return rc;
+    const bc_graph::Group &q = g->gr;
+    KParams p = p0;
+    p.sigma = q.sigma;
+    p.S = q.S;
+    p.ends = q.ends;
+    p.bigq = q.bigq;
+    p.gcodes = q.codes;
+    p.stride_codes = (size_t)q.code_words;
+    p.code_words = q.code_words;
+    p.nbits = q.nb;
+    p.stride_nb = 3 * (size_t)g->nb_words;
+    p.nb_words = g->nb_words;
+    p.sbits = q.sbits;
+    p.stride_sb = (size_t)g->sb_words;
+    p.sb_words = g->sb_words;
+    p.fb_words = 0;
+    bcgroup::GParams gp;
+    gp.groups = q.G;
+    gp.ctl = q.ctl;
+    CK(cudaMemsetAsync(q.ctl, 0, (size_t)q.G * bcgroup::CTL_WORDS * 8, st));
+    void *args[] = {&p, &gp};
+    cudaLaunchConfig_t lc{};
+    lc.gridDim = dim3(q.grid);
+    lc.blockDim = dim3(q.nt);
+    lc.dynamicSmemBytes = 0;
+    lc.stream = st;
+    cudaLaunchAttribute attr[2];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    int na = 1;
+    if (g->l2win.num_bytes) {
+        attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[1].val.accessPolicyWindow = g->l2win;
+        na = 2;
+    }
+    lc.attrs = attr;
+    lc.numAttrs = na;
+    CK(cudaLaunchKernelExC(&lc, bcgroup::group_kernel_fn(q.nt), args));
+    CK(cudaGetLastError());
+    g->launches++;
+    g->bc_launches++;
+    g->last_inflight = std::max(g->last_inflight, q.G);
+    return BC_OK;
 }
 
 static int launch_batch(bc_graph *g, const bcbatch::BParams &bp0, cudaStream_t st) {
@@ -477,6 +626,7 @@ extern "C" void bc_destroy(bc_graph *g) {
     if (g->done) cudaEventSynchronize(g->done);
     free_workspace(g);
     free_batch(g);
+    free_group(g);
     if (g->l2win.num_bytes) {
         cudaCtxResetPersistingL2Cache();
         cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
@@ -645,7 +795,7 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     if (o->n_samps < 1 || o->n_samps > 8192) return fail(BC_EINVAL, "n_samps must be in [1, 8192]");
     if (o->alpha < 0 || o->beta < 0 || o->ep_min_frontier < 0 || o->inflight < 0 || !(o->gamma >= 0) ||
         o->seq_max_deg < 0 || o->warp_max_deg < 0 || o->level_store < 0 || o->level_store > 3 ||
-        o->engine < 0 || o->engine > 2 || o->batch_levels < 0 || o->batch_levels > bcbatch::MAX_LCAP ||
+        o->engine < 0 || o->engine > 3 || o->group_ctas < 0 || o->batch_levels < 0 || o->batch_levels > bcbatch::MAX_LCAP ||
         o->hub_chunk < 0)
         return fail(BC_EINVAL, "invalid parameter");
     if (o->block_threads != 0 && o->block_threads != 128 && o->block_threads != 256 &&
@@ -655,6 +805,7 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
     if (g->done) CK(cudaEventSynchronize(g->done));
     const bc_options old = g->opt;
     g->opt = *o;
+    free_group(g);  // re-sized on its next use
     int rc = configure(g);
     if (rc) {
         g->opt = old;
@@ -727,6 +878,7 @@ static KParams base_params(bc_graph *g, double *d_bc) {
 
 static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
     if (p0.k <= 0) return BC_OK;
+    if (group_wanted(g, p0)) return launch_group(g, p0, st);
     KParams p = p0;
     // An EP level needs a frontier of >= ep_min_frontier (Alg. 5 guard) or > beta
     // (Alg. 4) vertices; when no frontier can be that large, the work-efficient-only

@@ -1,0 +1,48 @@
+// bc_group.cuh -- the group engine: G groups of CTAs, each group traversing one source at a
+// time.
+//
+// The same per-source Brandes computation as bc_kernel (Alg. 1-3, work-efficient
+// levels only), with a source's levels spread over the C = grid / G CTAs of its group
+// instead of one CTA.  Only G sources are in flight, so their per-source state (sigma /
+// omega f64[n], 2-bit level codes, successor bits) can stay in L2 on graphs whose state is
+// far too large for the ~300 sources the per-source engine keeps in flight (n = 2^22:
+// 32 MB of sigma per source).  Undirected graphs only (2-bit level codes).
+//
+// Forward level L (one group barrier per level):
+//   (a) every CTA expands the level-L vertices IT owns (row_pass of bc_kernels.cuh: fused
+//       discovery + sigma pull); discoveries set the 2-bit code and a bit of the level's
+//       discovery bitmap (idempotent ORs, no winner election)
+//   (b) group barrier: level L+1 is complete
+//   (c) every CTA compacts the bitmap words it owns into S (one atomicAdd on the level's
+//       counter reserves its range) and goes straight on to expand them: no second barrier.
+// Ownership: vertex v < 32 C (the highest-degree vertices after the internal relabelling)
+// belongs to CTA v mod C, every other vertex to CTA (v / 32) mod C, so hubs spread over the
+// group.  Bitmaps are triple-buffered by level (marks of level L+3 may start before every
+// CTA has read level L+1's bits).  Backward level L: the level S[ends[L], ends[L+1]) is cut
+// in 32-vertex chunks over all warps of the group, one barrier per level.
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace bcdev {
+struct KParams;
+}
+
+namespace bcgroup {
+
+constexpr int CTL_WORDS = 32;  // u64 per group control block (256 B)
+
+struct GParams {
+    int groups;                  // G; group g owns CTAs [ceil(g T / G), ceil((g+1) T / G))
+    unsigned long long *ctl;     // [G][CTL_WORDS]: [0] barrier count, [8] next source index,
+                                 // [16..17] four int32 level counters (ring); zero at launch
+};
+
+// Kernel symbol for a block size (256 or 512 threads); launched cooperatively with
+// arguments (KParams, GParams).  KParams: sigma / S / ends / gcodes / nbits (3 buffers of
+// nb_words) / sbits are per GROUP (strides stride_n, stride_e, stride_codes, stride_nb,
+// stride_sb); bigq is per CTA (stride_big).
+const void *group_kernel_fn(int nt);
+
+}  // namespace bcgroup

@@ -152,6 +152,9 @@ struct Smem {
     long long idx;
     int cnt[3];           // level L appends at S[hi + cnt[L % 3]] (triple-buffered, see kernel)
     int nbig;             // rows queued for CTA-cooperative expansion in this tile
+    int gw0, gwn;         // row_pass chunk distribution: this CTA's first warp index, warps
+                          // sharing the pass (0 / NT/32, except in the group engine's backward)
+    int goff;             // group engine: this CTA's offset in the level being compacted
     CtaStats st;
     double red[NT / 32];  // block reduction scratch
     int wtot[NT / 32];    // per-warp totals (frontier compaction)
@@ -165,6 +168,7 @@ struct Smem {
 // Exact int32 distances in HBM (directed graphs, or graphs too large for SMEM codes).
 struct GlobalLevels {
     static constexpr int UNVISITED = INF;
+    static constexpr bool SPEC_GATHER = false;  // gathers wait for the probe (see GlobalCodes)
     static constexpr bool RESET_VERTICES = true;
     static constexpr bool BITMAP_DISCOVERY = false;
     __device__ __forceinline__ void mark(int, int) const {}
@@ -189,6 +193,10 @@ struct GlobalLevels {
 // as SmemCodes; discoveries are global atomicOr.
 struct GlobalCodes {
     static constexpr int UNVISITED = 0;
+    // Speculative gathers (issued beside the probe, one round trip per arc quad instead of
+    // two) were measured slower on B200 (c5ws 2491 -> 2983 ms, c5k group 2479 -> 3430 ms):
+    // the extra sector requests cost more than the latency they hide.
+    static constexpr bool SPEC_GATHER = false;
     static constexpr bool RESET_VERTICES = false;
     // Discovery without winner election: mark() is an idempotent OR (RED, no return)
     // and the level is rebuilt from the per-level bitmap (compact_level).
@@ -240,6 +248,7 @@ struct GlobalCodes {
 // 2-bit level codes in shared memory, undirected graphs only (see header).
 struct SmemCodes {
     static constexpr int UNVISITED = 0;
+    static constexpr bool SPEC_GATHER = false;  // shared-memory probes are cheap
     static constexpr bool RESET_VERTICES = false;
     static constexpr bool BITMAP_DISCOVERY = false;
     __device__ __forceinline__ void mark(int, int) const {}
@@ -526,7 +535,10 @@ __device__ __forceinline__ void row_pass(const int *__restrict__ S, int lo, int 
     constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     // Phase A: each warp walks its own 32-vertex chunks; no CTA barrier.
-    for (int base = lo + wid * 32; base < hi; base += NT) {
+    // (Pipelining the S / row-bound loads of the next chunks was measured neutral on B200:
+    // c4 728 -> 725 ms, c3 270 -> 274 ms; not kept.)
+    const int gstep = sm.gwn * 32;
+    for (int base = lo + (sm.gw0 + wid) * 32; base < hi; base += gstep) {
         const int i = base + lane;
         int v = -1, beg = 0, deg = 0;
         if (i < hi) {
@@ -643,7 +655,14 @@ __device__ __forceinline__ int compact_level(uint32_t *nb, int words, int *out, 
 
 // ------------------------------------------------------------------ forward
 
-template <bool DIR, int NT, class LV>
+// L1G: sigma / omega gathers through L1 (ld.ca) instead of L2 only (ld.cg).  Safe where
+// every entry a level gathers was written by plain stores of this SM or before an L1
+// invalidation (work-efficient-only kernels; the group engine's barriers): neighbouring
+// lanes then share sectors of local neighbours and hub entries in L1.  EP-capable kernels
+// keep ld.cg, since EP levels accumulate sigma with L2 atomics.
+__device__ __forceinline__ double ld_sig(const double *a, bool l1) { return l1 ? __ldca(a) : __ldcg(a); }
+
+template <bool DIR, int NT, class LV, bool L1G = false>
 __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S, int *bigq,
                            uint32_t *nb, uint32_t *sb, int L, int lo, int hi, Smem<NT> &sm,
                            Counters &c) {
@@ -656,7 +675,13 @@ __device__ void forward_we(const KParams &p, const LV &lv, double *sigma, int *S
     ab.unv = LV::UNVISITED;
     const ArcBits none_ab;
     auto probe = [&](int u) -> int { return lv.probe(u); };
-    auto pull = [&](int u, int k) -> double { return k == kprev ? __ldcg(&sigma[u]) : 0.0; };
+    auto pull = [&](int u, int k) -> double {
+        if (LV::SPEC_GATHER) {
+            const double sv = ld_sig(&sigma[u], L1G);
+            return k == kprev ? sv : 0.0;
+        }
+        return k == kprev ? ld_sig(&sigma[u], L1G) : 0.0;
+    };
     auto claim = [&](int u, int k) -> bool {
         if (LV::BITMAP_DISCOVERY) {
             // no winner election: idempotent OR of the code and of the level bitmap
@@ -803,7 +828,7 @@ __device__ __forceinline__ void finish_dependency(const KParams &p, double sw, d
     if (p.dbg_delta) p.dbg_delta[w] = delta;
 }
 
-template <int NT, class LV>
+template <int NT, class LV, bool L1G = false>
 __device__ void backward_we(const KParams &p, const LV &lv, double *sig_om, const int *S, int *bigq,
                             uint32_t *sb, int L, int lo, int hi, Smem<NT> &sm, Counters &c) {
     const int knext = LV::key(L + 1);
@@ -813,7 +838,13 @@ __device__ void backward_we(const KParams &p, const LV &lv, double *sig_om, cons
     ab.knext = knext;
     ab.unv = LV::UNVISITED;
     auto probe = [&](int v) -> int { return lv.probe(v); };
-    auto gather = [&](int v, int k) -> double { return k == knext ? __ldcg(&sig_om[v]) : 0.0; };
+    auto gather = [&](int v, int k) -> double {
+        if (LV::SPEC_GATHER && !sb) {
+            const double ov = ld_sig(&sig_om[v], L1G);
+            return k == knext ? ov : 0.0;
+        }
+        return k == knext ? ld_sig(&sig_om[v], L1G) : 0.0;
+    };
     auto noclaim = [&](int, int) -> bool { return false; };
     auto none = [&](int, int, bool) {};
     auto pre = [&](int w) -> double { return __ldcg(&sig_om[w]); };  // sigma[w], issued early
@@ -897,6 +928,8 @@ bc_kernel(KParams p) {
     if (threadIdx.x == 0) {
         sm.nbig = 0;
         sm.st = CtaStats{};
+        sm.gw0 = 0;
+        sm.gwn = NT / 32;
     }
 
     for (;;) {
@@ -928,7 +961,7 @@ bc_kernel(KParams p) {
             uint32_t *const nbl =
                 LV::BITMAP_DISCOVERY ? nb
                                      : ((nb && (long long)(hi - lo) * 4 >= p.sort_min) ? nb : nullptr);
-            if (!EPOK || mode == MODE_WE) forward_we<DIR, NT>(p, lv, sigma, S, bigq, nbl, sb, L, lo, hi, sm, c);
+            if (!EPOK || mode == MODE_WE) forward_we<DIR, NT, LV, !EPOK>(p, lv, sigma, S, bigq, nbl, sb, L, lo, hi, sm, c);
             else forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
             // (the level functions end with a barrier: every discovery is recorded)
             int nhi;
@@ -990,7 +1023,7 @@ bc_kernel(KParams p) {
             const long long t0 = clock64();
             // the forward's successor bits exist only if forward level Lb ran WE
             uint32_t *const sbl = (sb && (!EPOK || modes[Lb] == MODE_WE)) ? sb : nullptr;
-            if (!EPOK || bmode == MODE_WE) backward_we<NT>(p, lv, sigma, S, bigq, sbl, Lb, blo, bhi, sm, c);
+            if (!EPOK || bmode == MODE_WE) backward_we<NT, LV, !EPOK>(p, lv, sigma, S, bigq, sbl, Lb, blo, bhi, sm, c);
             else backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
             if (threadIdx.x == 0) {
                 const long long dt = clock64() - t0;

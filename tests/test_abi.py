@@ -58,6 +58,7 @@ int main(void){
          offsetof(bc_options, level_store), sizeof(bc_stats));
   printf("%zu %zu %zu\n", offsetof(bc_stats, sampling_ep), offsetof(bc_stats, inflight),
          offsetof(bc_stats, kernel_ms));
+  printf("%zu %zu %d\n", offsetof(bc_options, engine), offsetof(bc_options, group_ctas), BC_ENGINE_GROUP);
   return 0; }
 """
     import tempfile
@@ -69,7 +70,8 @@ int main(void){
         vals = [int(x) for x in subprocess.check_output([exe]).split()]
     O, S = _bc.bc_options, _bc.bc_stats
     assert vals == [ctypes.sizeof(O), O.gamma.offset, O.level_store.offset, ctypes.sizeof(S),
-                    S.sampling_ep.offset, S.inflight.offset, S.kernel_ms.offset]
+                    S.sampling_ep.offset, S.inflight.offset, S.kernel_ms.offset,
+                    O.engine.offset, O.group_ctas.offset, _bc.ENGINES["group"]]
 
 
 def test_default_options_are_the_papers(lib):
