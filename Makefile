@@ -32,3 +32,13 @@ clean:
 	rm -rf build $(PKG)/libbc.so $(PKG)/libgraphgen.so oracle/liboracle.so
 
 .PHONY: all clean
+
+# Tuning experiments: make variant VARIANT=name VFLAGS="-DBC_MINB512=3" builds
+# build/<name>/libbc.so (load it with BC_LIBBC=build/<name>/libbc.so).
+variant:
+	@mkdir -p build/$(VARIANT)
+	@for u in $(UNITS); do $(NVCC) $(NVFLAGS) $(VFLAGS) -c -o build/$(VARIANT)/$$u.o $(CSRC)/$$u.cu 2> build/$(VARIANT)/$$u.ptxas.log & done; wait
+	$(NVCC) $(ARCH) -shared -o build/$(VARIANT)/libbc.so $(UNITS:%=build/$(VARIANT)/%.o)
+	@cat build/$(VARIANT)/*.ptxas.log > build/$(VARIANT)/ptxas.log
+
+.PHONY: variant
