@@ -323,7 +323,8 @@ def run_ours(args):
     traffic = load_traffic(args.config, balg, st)
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
             "frac": achieved / hbm, "traffic": traffic, "peak_source": hbm_src,
-            "kernel": "bc_kernel (sampling + main launches per step)",
+            "kernel": " + ".join(n for b, n in ((1, "bc_kernel"), (2, "batch_kernel"), (4, "group_kernel"))
+                                 if st and st.get("engines", 1) & b) + " (sampling + main launches per step)",
             "kernel_ms_per_step": kms, "kernel_share_of_step": kms / (sum(step_ms) / len(step_ms)),
             "alg_bytes_per_step": balg,
             "alg_bytes_per_teps_edge": balg / (g.m * st["sources"]) if st and st["sources"] else None,

@@ -144,6 +144,9 @@ typedef struct bc_stats {
                                  backward WE, backward EP levels (device trace)               */
     int64_t batches;          /* batches of 64 sources run by the batched engine (0: not run) */
     int64_t batch_overflows;  /* ... of which exceeded batch_levels and were rerun per source */
+    int32_t engines;          /* engines the last compute call launched: bit 0 per-source
+                                 (bc_kernel), bit 1 batched, bit 2 group (group_kernel)      */
+    int32_t pad_;
 } bc_stats;
 
 /* Copy a CSR graph to `device` and allocate the per-source workspace.

@@ -50,7 +50,8 @@ class bc_stats(ctypes.Structure):
                 ("sigma_inexact", ctypes.c_int32), ("inflight", ctypes.c_int32),
                 ("kernel_launches", ctypes.c_int32), ("bc_kernel_launches", ctypes.c_int32),
                 ("kernel_ms", ctypes.c_double), ("phase_cycles", ctypes.c_int64 * 4),
-                ("batches", ctypes.c_int64), ("batch_overflows", ctypes.c_int64)]
+                ("batches", ctypes.c_int64), ("batch_overflows", ctypes.c_int64),
+                ("engines", ctypes.c_int32), ("pad_", ctypes.c_int32)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_}

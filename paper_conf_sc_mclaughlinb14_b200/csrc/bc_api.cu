@@ -126,6 +126,7 @@ struct bc_graph {
         long long *ovf_n = nullptr;
     } bt;
     int batch_ran = 0;       // the last compute call launched the batched engine
+    int engines = 0;         // engines launched by the last compute call (bc_stats.engines)
     // group engine (bc_group.cu); allocated on first use
     struct Group {
         int ready = 0, nt = 512, grid = 0, G = 0, code_words = 0, sb = 0;
@@ -508,6 +509,7 @@ static int launch_group(bc_graph *g, const KParams &p0, cudaStream_t st) {
     bcgroup::GParams gp;
     gp.groups = q.G;
     gp.ctl = q.ctl;
+    gp.own_block = g->perm ? 1 : 32;  // see bcgroup::Owned (measured per graph kind)
     CK(cudaMemsetAsync(q.ctl, 0, (size_t)q.G * bcgroup::CTL_WORDS * 8, st));
     void *args[] = {&p, &gp};
     cudaLaunchConfig_t lc{};
@@ -530,6 +532,7 @@ static int launch_group(bc_graph *g, const KParams &p0, cudaStream_t st) {
     CK(cudaGetLastError());
     g->launches++;
     g->bc_launches++;
+    g->engines |= 4;
     g->last_inflight = std::max(g->last_inflight, q.G);
     return BC_OK;
 }
@@ -584,6 +587,7 @@ static int launch_batch(bc_graph *g, const bcbatch::BParams &bp0, cudaStream_t s
     }
     g->launches++;
     g->bc_launches++;
+    g->engines |= 2;
     g->batch_ran = 1;
     g->last_inflight = std::max(g->last_inflight, g->bt.grid);
     return BC_OK;
@@ -908,6 +912,7 @@ static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
     g->last_inflight = std::max(g->last_inflight, grid);
     g->launches++;
     g->bc_launches++;
+    g->engines |= 1;
     CK(cudaGetLastError());
     return BC_OK;
 }
@@ -930,6 +935,7 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
     g->launches = g->bc_launches = 0;
     g->tev_used[0] = g->tev_used[1] = 0;
     g->batch_ran = 0;
+    g->engines = 0;
     KParams p = base_params(g, acc_bc);
     p.sources = d_sources;
     int rc = BC_OK;
@@ -1297,6 +1303,8 @@ extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {
     for (int q = 0; q < 4; ++q) st->phase_cycles[q] = (int64_t)h.phase_cycles[q];
     st->batches = (int64_t)h.batches;
     st->batch_overflows = (int64_t)h.batch_overflows;
+    st->engines = g->engines;
+    st->pad_ = 0;
     st->kernel_ms = 0.0;
     for (int i = 0; i < 2; ++i)
         if (g->tev_used[i]) {

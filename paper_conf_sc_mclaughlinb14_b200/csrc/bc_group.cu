@@ -37,21 +37,34 @@ __device__ __forceinline__ void group_sync(unsigned long long *bar, unsigned lon
 
 // Bits of the discovery bitmap `nb` owned by CTA r of C, as a list of items: item i < H
 // (H = min(C, words) "hub" words) is word i restricted to the vertices v = 32 i + j with
-// v mod C == r; item H + k is word r + C (k + 1), whole.  Items are in ascending vertex
-// order.
+// v mod C == r; the words after the hub words are dealt out in blocks of OB words, block
+// b to CTA b mod C; item H + k is word k mod OB of this CTA's (k / OB)-th block.  Items
+// are in ascending vertex order.  OB = GParams::own_block: 32 words (1,024 vertices) keeps
+// neighbouring ids -- the local neighbours of spatial / ring-ordered graphs -- with one
+// CTA and its L1 (c5ws 1604 -> 1547 ms); 1 word on degree-relabelled graphs, whose
+// consecutive ids have similar degrees (c5k: 32 words 2479 -> 2629 ms).
+// Levels whose per-CTA share is remembered for the backward (deeper levels -- only on
+// graphs of diameter > RCAP -- are cut in 32-vertex chunks over the whole group).
+constexpr int RCAP = 1024;
 struct Owned {
     const uint32_t *nb;
-    int words, r, C, H, items;
-    __device__ __forceinline__ Owned(const uint32_t *nb_, int words_, int r_, int C_)
-        : nb(nb_), words(words_), r(r_), C(C_) {
+    int words, r, C, OB, H, items;
+    __device__ __forceinline__ Owned(const uint32_t *nb_, int words_, int r_, int C_, int ob_)
+        : nb(nb_), words(words_), r(r_), C(C_), OB(ob_) {
         H = min(C, words);
-        const int wn = words > r ? (words - r - 1) / C : 0;
-        items = H + wn;
+        const int T = words - H, nbk = T / OB, rem = T % OB;
+        const int full = nbk > r ? (nbk - 1 - r) / C + 1 : 0;        // whole blocks owned
+        const int part = (rem > 0 && nbk % C == r) ? rem : 0;          // the ragged last block
+        items = H + full * OB + part;
     }
-    __device__ __forceinline__ int word(int i) const { return i < H ? i : r + C * (i - H + 1); }
+    __device__ __forceinline__ int word(int i) const {
+        if (i < H) return i;
+        const int k = i - H;
+        return H + (r + (k / OB) * C) * OB + (k % OB);
+    }
     __device__ __forceinline__ uint32_t bits(int i) const {
         if (i >= items) return 0u;
-        if (i >= H) return __ldcg(&nb[word(i)]);
+        if (i >= H) return __ldcg(&nb[word(i)]);  // (word order = item order)
         uint32_t m = 0u;
         int j = (int)(((long long)r - 32LL * i) % C);
         if (j < 0) j += C;
@@ -64,11 +77,11 @@ struct Owned {
 // reserved with one atomicAdd on *ctr; clears the owned whole words (hub words are cleared
 // later by rank 0, once every CTA has read them).  Returns this CTA's count; sets off.
 template <int NT>
-__device__ __forceinline__ int group_compact(uint32_t *nb, int words, int r, int C, int *out, int *ctr,
-                                             Smem<NT> &sm, int &off) {
+__device__ __forceinline__ int group_compact(uint32_t *nb, int words, int r, int C, int ob, int *out,
+                                             int *ctr, Smem<NT> &sm, int &off) {
     constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const Owned ow(nb, words, r, C);
+    const Owned ow(nb, words, r, C, ob);
     const int per = ((ow.items + NW - 1) / NW + 31) & ~31;  // items per warp, multiple of 32
     const int i0 = min(wid * per, ow.items), i1 = min(i0 + per, ow.items);
     int cnt = 0;
@@ -115,6 +128,7 @@ template <int NT>
 __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p, GParams gp) {
     constexpr int NW = NT / 32;
     __shared__ Smem<NT> sm;
+    __shared__ int2 s_reg[RCAP];  // this CTA's share of level L in S: (offset, count), L < RCAP
     const int T = gridDim.x, G = gp.groups;
     const int g = (int)((long long)blockIdx.x * G / T);
     const int b0 = (int)(((long long)g * T + G - 1) / G);
@@ -165,6 +179,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             lvl[1] = 0;
         }
         int mylo = 0, mycnt = r == 0 ? 1 : 0;  // this CTA's vertices of level L: S[mylo, +mycnt)
+        if (tid == 0) s_reg[0] = make_int2(mylo, mycnt);
         int prevlo = 0, prevcnt = 0;
         int startL = 0;                        // ends[L]
         int L = 0;
@@ -195,11 +210,12 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             }
             // (c) this CTA's part of level L+1, in vertex order, straight into S
             int off = 0;
-            const int cnt = group_compact<NT>(nbw_next, nbw, r, C, S + endL1, &lvl[(L + 1) & 3], sm, off);
+            const int cnt = group_compact<NT>(nbw_next, nbw, r, C, gp.own_block, S + endL1, &lvl[(L + 1) & 3], sm, off);
             prevlo = mylo;
             prevcnt = mycnt;
             mylo = endL1 + off;
             mycnt = cnt;
+            if (tid == 0 && L + 1 < RCAP) s_reg[L + 1] = make_int2(mylo, mycnt);
             startL = endL1;
             ++L;
         }
@@ -220,26 +236,34 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
         }
         // Stage 2 (Alg. 3).  Deepest level: delta = 0, omega = 1/sigma (in place), by owner.
         if (maxdepth >= 1) {
-            if (tid == 0) {
-                sm.gw0 = r * NW;  // backward levels: 32-vertex chunks over every warp of the group
-                sm.gwn = C * NW;
-            }
             for (int i = prevlo + tid; i < prevlo + prevcnt; i += NT) {
                 const int v = S[i];
                 sigma[v] = 1.0 / __ldcg(&sigma[v]);
             }
             group_sync(bar, target, C);
         }
+        // Backward levels: each CTA finishes the vertices it expanded in the forward (same
+        // ownership, same locality); levels >= RCAP in 32-vertex chunks over the group.
         for (int Lb = maxdepth - 1; Lb >= 1; --Lb) {
             const long long t0 = clock64();
-            const int blo = ends[Lb], bhi = ends[Lb + 1];
-            backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, blo, bhi, sm, c);
+            if (Lb < RCAP) {
+                const int2 rg = s_reg[Lb];
+                backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, rg.x, rg.x + rg.y, sm, c);
+            } else {
+                if (tid == 0) {
+                    sm.gw0 = r * NW;
+                    sm.gwn = C * NW;
+                }
+                __syncthreads();
+                backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, ends[Lb], ends[Lb + 1], sm, c);
+                __syncthreads();
+                if (tid == 0) {
+                    sm.gw0 = 0;
+                    sm.gwn = NW;
+                }
+            }
             group_sync(bar, target, C);
             if (r == 0 && tid == 0 && p.dbg_bcyc && Lb < p.dbg_max_levels) p.dbg_bcyc[Lb] = clock64() - t0;
-        }
-        if (tid == 0) {
-            sm.gw0 = 0;
-            sm.gwn = NW;
         }
         // Reset of this source's codes and successor bits (the bitmaps are clear already),
         // then the next source.

@@ -16,10 +16,11 @@
 //   (c) every CTA compacts the bitmap words it owns into S (one atomicAdd on the level's
 //       counter reserves its range) and goes straight on to expand them: no second barrier.
 // Ownership: vertex v < 32 C (the highest-degree vertices after the internal relabelling)
-// belongs to CTA v mod C, every other vertex to CTA (v / 32) mod C, so hubs spread over the
-// group.  Bitmaps are triple-buffered by level (marks of level L+3 may start before every
-// CTA has read level L+1's bits).  Backward level L: the level S[ends[L], ends[L+1]) is cut
-// in 32-vertex chunks over all warps of the group, one barrier per level.
+// belongs to CTA v mod C, the other vertices in blocks of own_block bitmap words dealt out
+// round-robin, so hubs spread over the group.  Bitmaps are triple-buffered by level (marks
+// of level L+3 may start before every CTA has read level L+1's bits).  Backward level L is
+// finished by the CTAs that expanded its vertices in the forward (same ownership), one
+// barrier per level.
 #pragma once
 
 #include <cstdint>
@@ -37,6 +38,7 @@ struct GParams {
     int groups;                  // G; group g owns CTAs [ceil(g T / G), ceil((g+1) T / G))
     unsigned long long *ctl;     // [G][CTL_WORDS]: [0] barrier count, [8] next source index,
                                  // [16..17] four int32 level counters (ring); zero at launch
+    int own_block;               // bitmap words per ownership block (>= 1), see Owned
 };
 
 // Kernel symbol for a block size (256 or 512 threads); launched cooperatively with

@@ -155,3 +155,20 @@ def test_auto_engine_picks_group_on_large_graphs(bcmod, oracle_mod):
     with bcmod.BCGraph.from_graph(g, ep_min_frontier=NO_EP) as bg:
         check_bc(bg, g, src, oracle_mod, nthreads=16)
         assert bg.stats()["inflight"] > 64
+
+
+@pytest.mark.parametrize("key", ["c5ws", "c5k"])
+def test_group_matches_per_source_on_many_sources(bcmod, key):
+    """Every BFS of 1,024 sources agrees between the engines: the traversal counters (levels,
+    reached vertices and arcs, DAG arcs) are exact integers, BC within 1e-9.  Races in the
+    group barrier / ownership / bitmap protocol show up here first."""
+    g = graph(key)
+    src = gg.CONFIGS[key].sources(g)[:1024]
+    out = {}
+    for eng in ("per_source", "group"):
+        with bcmod.BCGraph.from_graph(g, engine=eng, strategy="we") as bg:
+            bc = bg.compute(src)
+            st = bg.stats()
+            out[eng] = (bc, [st[k] for k in ("levels", "n_reached", "arcs_reached", "dag_arcs")])
+    assert out["group"][1] == out["per_source"][1]
+    assert rel_err(out["group"][0], out["per_source"][0]) <= BC_TOL

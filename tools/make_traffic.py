@@ -30,7 +30,7 @@ def main():
     kernels = 0
     for r in rows[2:]:
         d = dict(zip(h, r))
-        if "bc_kernel" not in d.get("Kernel Name", ""):
+        if not any(k in d.get("Kernel Name", "") for k in ("bc_kernel", "group_kernel", "batch_kernel")):
             continue
         kernels += 1
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
