@@ -100,7 +100,7 @@ typedef struct bc_options {
                                 memory (undirected graphs whose codes fit; else EINVAL),
                                 3 = 2-bit codes in HBM/L2 (undirected graphs)                  */
     int32_t warp_max_deg;    /* rows up to this degree are expanded by one warp, longer rows
-                                by the whole CTA.  0 = auto (16384)                            */
+                                by the whole CTA.  0 = auto (8192)                             */
     int32_t l2_persist;      /* 0 = auto (on), -1 = off: persisting-L2 access-policy window
                                 over the CSR arrays during traversal launches                  */
     int32_t sort_frontier;   /* 0 = auto, 1 = on, -1 = off: rebuild large BFS levels in vertex

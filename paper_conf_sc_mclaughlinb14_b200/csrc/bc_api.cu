@@ -129,7 +129,7 @@ struct bc_graph {
     int engines = 0;         // engines launched by the last compute call (bc_stats.engines)
     // group engine (bc_group.cu); allocated on first use
     struct Group {
-        int ready = 0, nt = 512, grid = 0, G = 0, code_words = 0, sb = 0;
+        int ready = 0, failed = 0, nt = 512, grid = 0, G = 0, code_words = 0, sb = 0;
         unsigned long long *ctl = nullptr;
         double *sigma = nullptr;
         int *S = nullptr, *ends = nullptr, *bigq = nullptr;
@@ -228,9 +228,11 @@ static int configure(bc_graph *g) {
         return fail(BC_EINVAL, "block_threads must be 0, 128, 256, 512 or 1024");
     // defaults from tools/sweep_rows.sh on B200 (c4: 110.7 -> 103.8 ms, c3 82 -> 79 ms):
     // one-thread rows keep 32 independent rows in flight per warp, which beats warp
-    // cooperation up to degree ~128; CTA cooperation only pays for rows > 16384
+    // cooperation up to degree ~128; CTA cooperation pays for rows > 8192 (re-swept with the
+    // group engine, tools/gpu/sweep_rows2.txt: c4 735.7 -> 731.7 ms, c5k 2335 -> 2195 ms;
+    // 2048 / 4096 lose on c4, 64 / 256 one-thread rows lose on c4)
     g->seq_max_deg = o.seq_max_deg > 0 ? o.seq_max_deg : 128;
-    g->warp_max_deg = std::max(g->seq_max_deg, o.warp_max_deg > 0 ? o.warp_max_deg : 16384);
+    g->warp_max_deg = std::max(g->seq_max_deg, o.warp_max_deg > 0 ? o.warp_max_deg : 8192);
     // Sorted frontiers: a level is rebuilt in vertex order from the per-level bitmap
     // when it holds >= sort_min vertices (the scan costs n/32 words, so small levels
     // keep their append order).
@@ -472,7 +474,7 @@ static bool group_eligible(const bc_graph *g, const KParams &p) {
 // batched engine 2.2x / 1.14x); on smaller graphs the per-source engine
 // (codes in shared memory, ~300 sources in flight) is faster (c4: 728 vs 1374 ms).
 static bool group_auto(const bc_graph *g) {
-    return g->opt.engine == BC_ENGINE_AUTO && !g->directed && g->n >= (1 << 21);
+    return g->opt.engine == BC_ENGINE_AUTO && !g->directed && g->n >= (1 << 21) && !g->gr.failed;
 }
 
 static bool group_wanted(const bc_graph *g, const KParams &p) {
@@ -882,7 +884,13 @@ static KParams base_params(bc_graph *g, double *d_bc) {
 
 static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
     if (p0.k <= 0) return BC_OK;
-    if (group_wanted(g, p0)) return launch_group(g, p0, st);
+    if (group_wanted(g, p0)) {
+        const int rc = launch_group(g, p0, st);
+        if (rc == BC_OK || g->opt.engine == BC_ENGINE_GROUP) return rc;
+        free_group(g);
+        g->gr.failed = 1;  // auto: e.g. no memory for the group workspace -> per-source engine
+        cudaGetLastError();
+    }
     KParams p = p0;
     // An EP level needs a frontier of >= ep_min_frontier (Alg. 5 guard) or > beta
     // (Alg. 4) vertices; when no frontier can be that large, the work-efficient-only
