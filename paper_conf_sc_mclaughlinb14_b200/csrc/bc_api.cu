@@ -512,6 +512,7 @@ static int launch_group(bc_graph *g, const KParams &p0, cudaStream_t st) {
     gp.groups = q.G;
     gp.ctl = q.ctl;
     gp.own_block = g->perm ? 1 : 32;  // see bcgroup::Owned (measured per graph kind)
+    if (const char *ob = getenv("BC_OWN_BLOCK")) gp.own_block = std::max(1, atoi(ob));  // tuning
     CK(cudaMemsetAsync(q.ctl, 0, (size_t)q.G * bcgroup::CTL_WORDS * 8, st));
     void *args[] = {&p, &gp};
     cudaLaunchConfig_t lc{};
