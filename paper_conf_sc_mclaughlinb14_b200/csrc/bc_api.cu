@@ -417,11 +417,11 @@ static void free_group(bc_graph *g) {
 // together, at least one; group_ctas > 0 fixes the CTAs per group instead.
 static int group_count(const bc_graph *g, int grid) {
     if (g->opt.group_ctas > 0) return std::max(1, std::min(grid, grid / g->opt.group_ctas));
-    // Auto, from the B200 sweep (kernel ms for 2,048 sources): the unskewed
-    // small world c5ws is fastest with 4 groups of 74 CTAs (1604 ms; 1 group 1918, 8 groups
-    // 1667), the skewed Kronecker c5k with groups of 9 CTAs (2479 ms; 18: 2873, 37: 3761,
-    // 4: 2505).  Skewed = internally relabelled by degree (want_reorder).
-    const int ctas = g->perm ? 9 : std::max(1, grid / 4);
+    // Auto, from the B200 sweeps (kernel ms for 2,048 sources): the unskewed
+    // small world c5ws is fastest with 4 groups of 74 CTAs (1509 ms; 148 CTAs 1590, 37:
+    // 1609), the skewed Kronecker c5k with groups of 12 CTAs (2103 ms; 9: 2149, 6: 2308,
+    // 18: 2552).  Skewed = internally relabelled by degree (want_reorder).
+    const int ctas = g->perm ? 12 : std::max(1, grid / 4);
     return std::max(1, std::min(grid, grid / ctas));
 }
 

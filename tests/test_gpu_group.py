@@ -141,7 +141,7 @@ def test_sampling_decision_matches_per_source(bcmod, oracle_mod):
 
 def test_auto_engine_picks_group_on_large_graphs(bcmod, oracle_mod):
     """Auto engine: group engine on n >= 2^21 when every level is work-efficient (4 groups
-    on the unskewed c5ws, groups of 9 CTAs on the relabelled c5k); per-source on c4."""
+    on the unskewed c5ws, groups of 12 CTAs on the relabelled c5k); per-source on c4."""
     for key, groups in (("c5ws", 4), ("c5k", None)):
         g = graph(key)
         src = gg.CONFIGS[key].sources(g)[:24]
