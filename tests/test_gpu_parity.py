@@ -439,3 +439,14 @@ def test_row_split_knobs(bcmod, oracle_mod, seq, warp):
             hub = int(np.argmax(g.degrees()))
             check_source(bg, g, hub, oracle_mod)
             check_source(bg, g, 3 if src is None else int(src[0]), oracle_mod)
+
+
+@pytest.mark.parametrize("strategy", STRATS)
+def test_fig1_consistent_golden(bcmod, oracle_mod, strategy):
+    """The CUDA path on the hand-derived Figure 1 fixture (tests/golden/)."""
+    import golden_io
+    g, want = golden_io.load("fig1_consistent.txt")
+    with bcmod.BCGraph.from_graph(g, strategy=strategy) as bg:
+        for s in range(g.n):
+            check_source(bg, g, s, oracle_mod)
+        assert rel_err(bg.compute(None), want) < 1e-12

@@ -236,3 +236,22 @@ def test_empty_and_isolated(oracle_mod):
     r = oracle_mod.single_source(g, 2)
     assert r["num_levels"] == 1 and r["n_reached"] == 1
     assert np.all(oracle_mod.bc(gg.path_graph(5), np.zeros(0, dtype=np.int32)) == 0)
+
+
+# ------------------------------------------------------------- golden fixtures
+
+
+def test_fig1_consistent_golden(oracle_mod):
+    """tests/golden/fig1_consistent.txt: hand-derived Eq. (1) values on a graph that
+    satisfies the Figure 1 prose."""
+    import golden_io
+    g, want = golden_io.load("fig1_consistent.txt")
+    got = oracle_mod.bc(g)
+    assert np.array_equal(got, want)
+    # the prose itself: 4 (index 3) scores highest; 8 and 9 score zero (P:72)
+    assert int(np.argmax(got)) == 3 and got[7] == 0 and got[8] == 0
+    # P:110: BFS from 4 has second frontier {1, 3, 5, 6}; P:72: 5 -> 9 is 5-7-9
+    r4 = oracle_mod.single_source(g, 3)
+    assert sorted(np.flatnonzero(r4["d"] == 1) + 1) == [1, 3, 5, 6]
+    r5 = oracle_mod.single_source(g, 4)
+    assert r5["d"][8] == 2 and r5["sigma"][8] == 1 and r5["d"][6] == 1
