@@ -6,11 +6,18 @@
 One STEP = one complete betweenness-centrality computation of the workload's
 source set (all of SURVEY §8(a): Alg. 5 sampling phase, decision, forward +
 backward traversal of every source, BC accumulation, halving) plus, for N > 1,
-the single NCCL all-reduce of the per-GPU BC vectors.  The default
-workload is configs[3] of BASELINE.json -- Graph500 Kronecker scale 18, edge
-factor 16, 16,384 sources -- the configuration the metric is quoted on at
-1/2/4/8 GPUs.  Scaling is weak: every rank processes 16,384 sources of its own
-(--scaling strong splits one 16,384-source set instead).
+the single NCCL all-reduce of the per-GPU BC vectors -- the step is
+`distributed.bc_step`, the same function the multi-process gloo tests drive.  The
+default workload is configs[3] of BASELINE.json -- Graph500 Kronecker scale 18,
+edge factor 16, 16,384 sources -- the configuration the metric is quoted on at
+1/2/4/8 GPUs.  Scaling is STRONG by default: the fixed 16,384-source set is split
+over the N GPUs (--scaling weak gives every GPU a set of that size instead).
+
+Multi-GPU: `python bench.py --gpus N` re-executes itself under torch.distributed.run
+with N ranks (one per GPU) when no torchrun environment is present, and exits with
+an error if fewer than N GPUs are visible.  The ≥7x scaling target of north_star is
+`python bench.py --gpus 8 --config c5k --steps 2` against `--gpus 1` (65,536 sources
+in both runs).
 
 Timing: inputs resident in HBM; L2 flushed (256 MiB write)
 before every timed step; CUDA events on the launching stream; barrier +
@@ -62,26 +69,48 @@ def peaks():
 
 
 def make_workload(cfg_key: str, world: int, rank: int, scaling: str, k_override: int = 0):
+    """(config, graph, total source list, this rank's shard).
+
+    strong (default): the config's fixed source list (BASELINE: 16,384 sources for c4 and
+    65,536 for c5 "at 1/2/4/8 GPUs"; all n for the exact-BC configs), split over the ranks.
+    weak: every rank gets a list of the config's size (world x as many sources in total).
+    k_override (--sources K): a bounded prefix of the list -- K in total (strong) or per
+    rank (weak)."""
     from paper_conf_sc_mclaughlinb14_b200 import graphgen as gg
     from paper_conf_sc_mclaughlinb14_b200.distributed import shard_sources
     cfg = gg.CONFIGS[cfg_key]
     g = cfg.graph()
-    if k_override:                        # --sources: a bounded prefix of the workload
+    if k_override:
         import dataclasses
         cfg = dataclasses.replace(cfg, k=k_override)
     if cfg.k is None:                     # exact BC: all vertices
         total = np.arange(g.n, dtype=np.int32)
-        local = shard_sources(total, rank, world, seed=cfg.seed)
-        per_rank = None
     elif scaling == "weak":
-        per_rank = cfg.k
         total = gg.sample_sources(g, min(cfg.k * world, int((g.degrees() > 0).sum())), cfg.seed + 7)
-        local = shard_sources(total, rank, world, seed=cfg.seed)
     else:
         total = cfg.sources(g)
-        local = shard_sources(total, rank, world, seed=cfg.seed)
-        per_rank = None
+    local = shard_sources(total, rank, world, seed=cfg.seed)
     return cfg, g, total, local
+
+
+def launch_ranks(args) -> int:
+    """--gpus N > 1 without a torchrun environment: re-exec this command under
+    torch.distributed.run with N ranks (one per GPU, rendezvous on 127.0.0.1)."""
+    import socket
+    import subprocess
+    import torch
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        log(f"--gpus {args.gpus} but only {have} CUDA device(s) visible: refusing to time fewer GPUs")
+        return 2
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    log("launching", " ".join(cmd[2:6]), "...")
+    return subprocess.call(cmd)
 
 
 # ---------------------------------------------------------------- clocks
@@ -220,14 +249,37 @@ def workload_config(cfg, g, total, world, args):
     return {"workload": f"{cfg.key}: {desc}", "graph": g.name, "n": g.n, "m": g.m,
             "sources_total": int(total.size), "sources_per_gpu": int(math.ceil(total.size / world)),
             "strategy": args.strategy, "options": bench_options(args),
-            "parallelism": f"sources split over {world} GPU(s)",
+            "parallelism": f"dp{world}: CSR replicated, sources split over {world} GPU(s), "
+                           f"one fp64 all-reduce per step" if world > 1 else "dp1",
             "l2": "flushed before every timed step (256 MiB write)", "seed": cfg.seed}
+
+
+def measure_l2_peak(dev, mib: int = 16, reps: int = 50):
+    """L2 bandwidth ceiling measured live: device copies between two `mib` MiB buffers
+    (a 2 x mib MiB working set that stays in L2), read + write bytes, best of 10."""
+    import torch
+    a = torch.ones(mib << 20, dtype=torch.uint8, device=dev)
+    b = torch.empty_like(a)
+    for _ in range(5):
+        b.copy_(a)
+    best = 0.0
+    for _ in range(10):
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(reps):
+            b.copy_(a)
+        e1.record()
+        e1.synchronize()
+        best = max(best, 2.0 * a.numel() * reps / (e0.elapsed_time(e1) / 1e3) / 1e9)
+    return best
 
 
 def run_ours(args):
     import torch
     import torch.distributed as dist
     import paper_conf_sc_mclaughlinb14_b200 as bcm
+    from paper_conf_sc_mclaughlinb14_b200 import distributed as bdist
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -241,7 +293,7 @@ def run_ours(args):
 
     t0 = time.time()
     cfg, g, total, local = make_workload(args.config, world, rank, args.scaling, args.sources)
-    log(f"rank {rank}: graph {g.name} n={g.n} m={g.m} local sources {local.size} "
+    log(f"rank {rank}: graph {g.name} n={g.n} m={g.m} sources {total.size} total, {local.size} local "
         f"(gen {time.time() - t0:.1f}s)")
     bg = bcm.BCGraph.from_graph(g, device=local_rank, **bench_options(args))
     stream = torch.cuda.Stream(dev)
@@ -250,10 +302,9 @@ def run_ours(args):
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
     def step():
+        # THE multi-GPU step (distributed.bc_step): this rank's shard, then one all-reduce
         with torch.cuda.stream(stream):
-            bg.compute_device(d_src, out, stream=stream)
-            if world > 1:
-                dist.all_reduce(out)
+            bdist.bc_step(lambda o: bg.compute_device(d_src, o, stream=stream), out)
 
     def barrier():
         torch.cuda.synchronize(dev)
@@ -291,18 +342,30 @@ def run_ours(args):
         dist.all_reduce(T, op=dist.ReduceOp.MAX)
     T = float(T.item())
     value = g.m * total.size * args.steps / T / 1e9
+    # BC self-check on the last step's reduced vector (any size):
+    # sum_v BC(v) = h * sum_s sum_{t reachable} (d(s,t) - 1), from the kernels' counters
+    h = 1.0 if g.directed else 0.5
+    cnt = torch.tensor([float(st["dist_sum"] - st["n_reached"] + st["sources"])], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(cnt)
+    want = h * float(cnt.item())
+    got = float(out.sum().item())
+    selfcheck = {"sum_bc": got, "h_sum_d_minus_1": want,
+                 "rel_err": abs(got - want) / max(abs(want), 1.0)}
 
     # -------- e2e: host-buffer C-ABI call (sources H2D and BC D2H inside the region)
     host_src = torch.from_numpy(local).pin_memory()
     host_bc = torch.empty(g.n, dtype=torch.float64).pin_memory()
+    dv = torch.empty(g.n, dtype=torch.float64, device=dev)
     e2e_ms = []
-    for it in range(args.warmup + args.steps):
+    e2e_steps = args.steps if args.e2e_steps is None else args.e2e_steps
+    for it in range(args.warmup + e2e_steps):
         flush.fill_(1)
         barrier()
         t0 = time.perf_counter()
         bcm.bc_compute(bg.handle, host_src.numpy(), host_bc.numpy())
         if world > 1:
-            dv = host_bc.to(dev, non_blocking=True)
+            dv.copy_(host_bc, non_blocking=True)
             dist.all_reduce(dv)
             host_bc.copy_(dv)
             torch.cuda.synchronize(dev)
@@ -312,47 +375,57 @@ def run_ours(args):
     Te = torch.tensor([sum(e2e_ms) / 1e3], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(Te, op=dist.ReduceOp.MAX)
-    e2e_value = g.m * total.size * args.steps / float(Te.item()) / 1e9
+    e2e_value = g.m * total.size * len(e2e_ms) / float(Te.item()) / 1e9
     h2d = 4 * local.size + (8 * g.n if world > 1 else 0)
     d2h = 8 * g.n * (2 if world > 1 else 1)
 
-    # -------- roofline of the dominant kernel (bc_kernel): algorithmic bytes / its event time
+    # -------- roofline of the dominant kernel: algorithmic bytes / its event time
     kms = sum(kern_ms) / max(1, len(kern_ms))
     balg = sum(bytes_alg) / max(1, len(bytes_alg))
     achieved = balg / (kms / 1e3) / 1e9 if kms > 0 else 0.0
-    traffic = load_traffic(args.config, balg, st)
+    tr = load_traffic(args.config, balg, kms)
+    l2peak = measure_l2_peak(dev)
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-            "frac": achieved / hbm, "traffic": traffic, "peak_source": hbm_src,
+            "frac": achieved / hbm, "traffic": tr["traffic"], "peak_source": hbm_src,
+            "traffic_source": tr["source"],
             "kernel": " + ".join(n for b, n in ((1, "bc_kernel"), (2, "batch_kernel"), (4, "group_kernel"))
                                  if st and st.get("engines", 1) & b) + " (sampling + main launches per step)",
             "kernel_ms_per_step": kms, "kernel_share_of_step": kms / (sum(step_ms) / len(step_ms)),
             "alg_bytes_per_step": balg,
             "alg_bytes_per_teps_edge": balg / (g.m * st["sources"]) if st and st["sources"] else None,
-            "model": "SURVEY 8(d): B(s) = 20n + 16 A_R + 24 D + 64 n_R per source"}
+            "model": "SURVEY 8(d): B(s) = 20n + 16 A_R + 24 D + 64 n_R per source",
+            "l2": {"peak_gbs": l2peak,
+                   "peak_source": "measured live: device copy over a 2 x 16 MiB L2-resident working set",
+                   "achieved_gbs": tr["l2_gbs"],
+                   "frac": (tr["l2_gbs"] / l2peak) if tr["l2_gbs"] else None,
+                   "source": tr["source"]}}
 
     result = None
-    if rank == 0:
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
         cores = len(os.sched_getaffinity(0))
-        cpu = None
-        if not args.no_cpu_baseline and world == 1:
-            v, k, dt = time_oracle(g, local, args.cpu_budget, cores)
-            cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
-                   "sample": f"first {k} of the {local.size} workload sources ({dt:.1f}s on {cores} threads)"}
+        v, k, dt = time_oracle(g, total, args.cpu_budget, cores)
+        cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"first {k} of the {total.size} workload sources ({dt:.1f}s on {cores} threads)"}
+    if world > 1:
+        dist.barrier(device_ids=[local_rank])        # ranks wait for rank 0's oracle leg
+    if rank == 0:
         result = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * T / args.steps, "higher_is_better": True,
             "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": workload_config(cfg, g, total, world, args),
             "e2e": {"value": e2e_value, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
-                    "d2h_bytes_per_step": int(d2h)},
+                    "d2h_bytes_per_step": int(d2h), "steps": len(e2e_ms)},
             "roofline": roof,
             "cpu_baseline": cpu,
             "clocks": clk.summary(),
             "gpu_launches": int(launches),
+            "selfcheck": selfcheck,
             "stats": {k2: st[k2] for k2 in ("sources", "levels", "we_levels", "ep_levels",
                                             "sampling_ep", "sampling_median", "inflight",
                                             "sigma_inexact", "arcs_scanned", "n_reached",
-                                            "arcs_reached", "dag_arcs")},
+                                            "arcs_reached", "dag_arcs", "dist_sum", "engines")},
             "paper_context": "398.63 MTEPS on 1x GTX Titan (Table III, smallworld); 24.13 GTEPS on "
                              "192x Tesla M2090 (Table IV, kron_g500-logn20)",
         }
@@ -363,17 +436,27 @@ def run_ours(args):
     return 0
 
 
-def load_traffic(cfg_key, balg, st):
-    """DRAM bytes per launch-step from the committed ncu capture, scaled by the
-    algorithmic bytes (profiles/traffic.json: dram bytes per algorithmic byte)."""
+def load_traffic(cfg_key, balg, kms):
+    """DRAM and L2 bytes per step SCALED from a committed ncu capture of the same config
+    (profiles/traffic.json: dram / lts bytes per algorithmic byte of that capture) -- not
+    measured in this run (an ncu replay cannot run inside the timed bench)."""
+    res = {"traffic": None, "l2_gbs": None, "source": None}
     p = os.path.join(ROOT, "profiles", "traffic.json")
     if not os.path.exists(p):
-        return None
+        return res
     try:
         d = json.load(open(p)).get(cfg_key)
-        return None if d is None else d["dram_bytes_per_alg_byte"] * balg
     except Exception:
-        return None
+        return res
+    if d is None:
+        return res
+    res["traffic"] = d["dram_bytes_per_alg_byte"] * balg
+    if d.get("lts_bytes_per_alg_byte") and kms > 0:
+        res["l2_gbs"] = d["lts_bytes_per_alg_byte"] * balg / (kms / 1e3) / 1e9
+    res["source"] = (f"scaled from ncu capture profiles/traffic.json[{cfg_key}] "
+                     f"({d.get('source')}, {d.get('sources')} sources): bytes per algorithmic byte x this run's "
+                     f"algorithmic bytes")
+    return res
 
 
 def main():
@@ -388,11 +471,14 @@ def main():
                     help="Alg. 5 EP guard (min frontier for an EP level); paper: 512")
     ap.add_argument("--paper-params", action="store_true",
                     help="use the paper's EP guard (512) instead of the B200-retuned one")
-    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--scaling", default="strong", choices=["weak", "strong"],
+                    help="strong (default): the config's fixed source set split over the GPUs; "
+                         "weak: the config's source count per GPU")
     ap.add_argument("--engine", default="auto", choices=["auto", "per_source", "batched", "group"],
                     help="source scheduling (include/bc.h BC_ENGINE_*)")
     ap.add_argument("--sources", type=int, default=0,
-                    help="sources per GPU (0 = the config's own count); bounds c5 runs")
+                    help="bounded prefix of the config's sources: total (strong) or per GPU (weak)")
+    ap.add_argument("--e2e-steps", type=int, default=None, help="timed e2e steps (default: --steps)")
     ap.add_argument("--cpu-budget", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
@@ -401,6 +487,8 @@ def main():
         args.warmup = 3
     if args.impl == "reference":
         return run_reference(args)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return launch_ranks(args)
     return run_ours(args)
 
 

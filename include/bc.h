@@ -61,11 +61,14 @@ enum {
 
 /* Execution engine (how sources are scheduled; results are the same up to fp64 rounding). */
 enum {
-    BC_ENGINE_AUTO = 0,       /* per-source engine, except that a SAMPLING run whose Alg. 5
-                                 decision is EP ("small-world": median depth < gamma*log2 n)
-                                 on a large (n >= 2^21) undirected graph with a skewed degree
-                                 distribution runs its main phase batched (measured faster
-                                 there only)                                   */
+    BC_ENGINE_AUTO = 0,       /* undirected graphs with n >= 2^21 whose launches run every
+                                 level work-efficiently (WE strategy, or SAMPLING with an EP
+                                 guard above n) use the GROUP engine; a SAMPLING run whose
+                                 Alg. 5 decision is EP on such a graph with a skewed degree
+                                 distribution (internally relabelled) runs its main phase on
+                                 the BATCHED engine; everything else (all graphs below 2^21,
+                                 directed graphs) runs on the PER-SOURCE engine.  Measured
+                                 choices, DESIGN.md §5d                                      */
     BC_ENGINE_PER_SOURCE = 1, /* one CTA per source (bc_kernel), every level WE or EP as the
                                  strategy chooses                                            */
     BC_ENGINE_BATCHED = 2,    /* undirected graphs: 64 sources per batch, level-synchronous
@@ -120,8 +123,10 @@ typedef struct bc_options {
     int32_t hub_chunk;       /* batched engine: minimum arcs per warp range when a BFS level's
                                 arcs are cut into equal warp ranges (rows of any length are
                                 split across ranges); 0 = auto 64                            */
-    int32_t group_ctas;      /* group engine: CTAs per group; 0 = auto (as many groups as keep
-                                their sigma + level codes + bitmaps within ~48 MB of L2)     */
+    int32_t group_ctas;      /* group engine: CTAs per group; 0 = auto (12 CTAs per group on
+                                degree-relabelled graphs, else 4 groups; B200 sweeps,
+                                DESIGN.md §5d).  bc_default_options sets every field, this
+                                one included                                                  */
 } bc_options;
 
 typedef struct bc_stats {
@@ -147,6 +152,9 @@ typedef struct bc_stats {
     int32_t engines;          /* engines the last compute call launched: bit 0 per-source
                                  (bc_kernel), bit 1 batched, bit 2 group (group_kernel)      */
     int32_t pad_;
+    int64_t dist_sum;         /* sum over sources s of sum_t d(s,t) over the reached t: with
+                                 n_reached and sources it gives the self-check
+                                 sum_v BC(v) = h (dist_sum - n_reached + sources) */
 } bc_stats;
 
 /* Copy a CSR graph to `device` and allocate the per-source workspace.
@@ -174,8 +182,12 @@ BC_API int bc_compute(bc_graph *g, const int32_t *sources, int64_t num_sources, 
 /* Same, device in / device out, asynchronous on `cuda_stream` (a cudaStream_t; NULL =
  * legacy default stream).  d_sources is DEVICE int32[k] or NULL (all n vertices); d_bc is
  * DEVICE double[n], OVERWRITTEN with the (halved if undirected) scores of these sources.
- * Sources are NOT range-checked on the device (caller's responsibility). Summing the
- * outputs of disjoint source lists gives the BC of their union (multi-GPU). */
+ * k = 0 with a non-NULL d_sources (never read) => d_bc all zero; NULL always means all n
+ * vertices, whatever k says (an empty device tensor must be passed as a non-NULL pointer:
+ * the Python binding does so).  Sources are NOT range-checked on the device (caller's
+ * responsibility).  Summing the outputs of disjoint source lists gives the BC of their
+ * union (multi-GPU) -- unless `extrapolate` is set, which scales each call by its
+ * own n/k (apply the estimator once, after the sum, instead: distributed.bc_distributed). */
 BC_API int bc_compute_device(bc_graph *g, const int32_t *d_sources, int64_t k, double *d_bc,
                       void *cuda_stream);
 

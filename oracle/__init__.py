@@ -79,6 +79,8 @@ def bc(g, sources: Optional[np.ndarray] = None, nthreads: int = 1, variant: str 
     out = np.zeros(g.n, dtype=np.float64)
     src = None if sources is None else np.ascontiguousarray(sources, dtype=np.int32)
     k = 0 if src is None else src.size
+    if src is not None and k == 0:
+        return out  # an empty source list: the empty sum (never "all vertices")
     f = lib.oracle_bc if variant == "pull" else lib.oracle_bc_push
     rc = f(g.n, _p(ro, _i64p), _p(col, _i32p), int(g.directed), _p(src, _i32p), k,
            _p(out, _f64p), int(nthreads))

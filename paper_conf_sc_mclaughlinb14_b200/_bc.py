@@ -51,7 +51,7 @@ class bc_stats(ctypes.Structure):
                 ("kernel_launches", ctypes.c_int32), ("bc_kernel_launches", ctypes.c_int32),
                 ("kernel_ms", ctypes.c_double), ("phase_cycles", ctypes.c_int64 * 4),
                 ("batches", ctypes.c_int64), ("batch_overflows", ctypes.c_int64),
-                ("engines", ctypes.c_int32), ("pad_", ctypes.c_int32)]
+                ("engines", ctypes.c_int32), ("pad_", ctypes.c_int32), ("dist_sum", ctypes.c_int64)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_}
@@ -265,6 +265,10 @@ class BCGraph:
         """sources: int32 CUDA tensor or None; out: float64 CUDA tensor [n]; async."""
         k = self.n if sources is None else int(sources.numel())
         sp = None if sources is None else sources.data_ptr()
+        if sources is not None and k == 0:
+            # an empty tensor has data_ptr() == 0, which the C ABI reads as "all n vertices";
+            # k = 0 with any non-NULL pointer (never dereferenced) yields an all-zero BC
+            sp = out.data_ptr()
         st = None if stream is None else stream.cuda_stream
         bc_compute_device(self.handle, sp, k, out.data_ptr(), st)
         return out

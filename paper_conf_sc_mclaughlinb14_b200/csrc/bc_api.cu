@@ -14,6 +14,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <mutex>
 #include <new>
 #include <vector>
 
@@ -52,6 +53,42 @@ struct DeviceGuard {
     }
 };
 
+// The persisting-L2 carve-out (cudaLimitPersistingL2CacheSize) is device-global state
+// shared by every handle on a device.  Handles register while they use a window; the
+// limit only grows while any handle holds it, and is reset (persisting lines released,
+// limit 0) when the last holder on the device lets go.
+struct L2Share {
+    int users = 0;
+    size_t carve = 0;
+};
+std::mutex g_l2_mu;
+L2Share g_l2[128];
+
+cudaError_t l2_acquire(int dev, size_t carve, bool held) {
+    std::lock_guard<std::mutex> lk(g_l2_mu);
+    L2Share &sh = g_l2[dev & 127];
+    if (!held) sh.users++;
+    if (carve > sh.carve) {
+        const cudaError_t e = cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve);
+        if (e != cudaSuccess) {
+            if (!held) sh.users--;
+            return e;
+        }
+        sh.carve = carve;
+    }
+    return cudaSuccess;
+}
+
+void l2_release(int dev) {
+    std::lock_guard<std::mutex> lk(g_l2_mu);
+    L2Share &sh = g_l2[dev & 127];
+    if (sh.users > 0 && --sh.users == 0) {
+        cudaCtxResetPersistingL2Cache();
+        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
+        sh.carve = 0;
+    }
+}
+
 }  // namespace
 
 struct bc_graph {
@@ -80,6 +117,7 @@ struct bc_graph {
     char *graph_buf = nullptr;          // ro | col | src
     size_t csr_bytes = 0, graph_bytes = 0;
     cudaAccessPolicyWindow l2win{};     // persisting-L2 window over the CSR (num_bytes 0 = off)
+    bool l2_held = false;               // registered as a user of the device's carve-out (L2Share)
     int *ro = nullptr, *col = nullptr, *src = nullptr;
     int *iro = nullptr, *icol = nullptr, *isrc = nullptr;
     // internal relabelling (see want_reorder): perm[old] = new; NULL = identity
@@ -139,6 +177,7 @@ struct bc_graph {
 
 extern "C" void bc_default_options(bc_options *o) {
     if (!o) return;
+    memset(o, 0, sizeof(*o));  // every field (and any padding) defined, whatever the caller left
     o->strategy = BC_STRATEGY_SAMPLING;
     o->alpha = 768;
     o->beta = 512;
@@ -159,6 +198,7 @@ extern "C" void bc_default_options(bc_options *o) {
     o->engine = BC_ENGINE_AUTO;
     o->batch_levels = 0;
     o->hub_chunk = 0;
+    o->group_ctas = 0;
 }
 
 extern "C" const char *bc_last_error(void) { return g_err; }
@@ -252,6 +292,10 @@ static int configure(bc_graph *g) {
     // Persisting-L2 window over the CSR (plus src[] when EP levels can run): every
     // in-flight source re-reads the same rows, while sigma/omega gathers stream.
     g->l2win = cudaAccessPolicyWindow{};
+    if (o.l2_persist < 0 && g->l2_held) {  // window switched off: stop holding the carve-out
+        l2_release(g->device);
+        g->l2_held = false;
+    }
     if (o.l2_persist >= 0 && g->graph_buf) {
         int max_persist = 0, max_win = 0;
         CK(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, g->device));
@@ -260,7 +304,8 @@ static int configure(bc_graph *g) {
             const size_t span = o.strategy == BC_STRATEGY_WE ? g->csr_bytes : g->graph_bytes;
             const size_t want = std::min<size_t>(span, (size_t)max_win);
             const size_t carve = std::min<size_t>(want, (size_t)max_persist);
-            CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve));
+            CK(l2_acquire(g->device, carve, g->l2_held));
+            g->l2_held = true;
             g->l2win.base_ptr = g->graph_buf;
             g->l2win.num_bytes = want;
             g->l2win.hitRatio = (float)((double)carve / (double)want);
@@ -284,13 +329,19 @@ static int configure(bc_graph *g) {
     return BC_OK;
 }
 
+// Per-slot capacity of bigq (rows queued for CTA-cooperative expansion): a level queues at
+// most nnz / (warp_max + 1) rows, warp_max being the EFFECTIVE threshold configure() derived
+// (max(seq_max_deg, warp_max_deg)), so the stride must follow every change of either knob.
+static size_t big_stride(const bc_graph *g) {
+    return (((size_t)g->nnz / ((size_t)g->warp_max_deg + 1) + 2) + 31) & ~(size_t)31;
+}
+
 static int alloc_workspace(bc_graph *g) {
     free_workspace(g);
     g->stride_n = (size_t)std::max(g->n, 1);
     g->stride_n = (g->stride_n + 31) & ~(size_t)31;  // 128-byte aligned slots
     g->stride_e = g->stride_n + 32;
-    // a level queues at most nnz / (warp_max + 1) rows for CTA-cooperative expansion
-    g->stride_big = (((size_t)g->nnz / ((size_t)g->warp_max_deg + 1) + 2) + 31) & ~(size_t)31;
+    g->stride_big = big_stride(g);
     const int occ = std::max(g->cfg_we.per_sm, g->cfg_ep.per_sm) * g->num_sms;
     int want = g->opt.inflight > 0 ? std::min(g->opt.inflight, occ) : occ;
     size_t free_b = 0, total_b = 0;
@@ -634,10 +685,7 @@ extern "C" void bc_destroy(bc_graph *g) {
     free_workspace(g);
     free_batch(g);
     free_group(g);
-    if (g->l2win.num_bytes) {
-        cudaCtxResetPersistingL2Cache();
-        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
-    }
+    if (g->l2_held) l2_release(g->device);  // the last holder on the device resets the carve-out
     cudaFree(g->graph_buf);
     cudaFree(g->perm);
     cudaFree(g->bc_tmp);
@@ -820,8 +868,10 @@ extern "C" int bc_set_options(bc_graph *g, const bc_options *o) {
         return rc;
     }
     const int old_slots = g->slots;
+    // bigq follows the effective row-split threshold (seq_max_deg AND warp_max_deg): a
+    // smaller threshold queues more rows per level, so the workspace must grow with it
     const int realloc = o->inflight != old.inflight || o->level_store != old.level_store ||
-                        o->block_threads != old.block_threads || o->warp_max_deg != old.warp_max_deg ||
+                        o->block_threads != old.block_threads || big_stride(g) != g->stride_big ||
                         o->sort_frontier != old.sort_frontier || o->succ_bits != old.succ_bits;
     if (realloc) {
         rc = alloc_workspace(g);
@@ -1314,6 +1364,7 @@ extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {
     st->batch_overflows = (int64_t)h.batch_overflows;
     st->engines = g->engines;
     st->pad_ = 0;
+    st->dist_sum = (int64_t)h.dist_sum;
     st->kernel_ms = 0.0;
     for (int i = 0; i < 2; ++i)
         if (g->tev_used[i]) {

@@ -28,6 +28,7 @@ __device__ __forceinline__ size_t sidx(const BParams &, int b, int v) { return (
 
 struct Cnt {  // per-lane counters of one batch (32-bit: a batch is ~10^8 events per warp at most)
     unsigned reached = 0, ar = 0, dag = 0, sc = 0;
+    unsigned long long dsum = 0;  // sum of d_b(u) over the (u, b) pairs this lane counted
     int inexact = 0;
 };
 
@@ -292,6 +293,7 @@ __device__ __forceinline__ void process_range(const BParams &p, const Level &lv,
             c.dag += (unsigned)__popcll(m);
             if (ok && a == rs) {  // first arc of the row: per-row statistics
                 c.reached += (unsigned)__popcll(f);
+                c.dsum += (unsigned long long)L * (unsigned long long)__popcll(f);
                 c.ar += (unsigned)__popcll(f) * (unsigned)(re - rs);
                 wor |= f;
             }
@@ -382,10 +384,10 @@ __global__ void __launch_bounds__(NT, 768 / NT) batch_kernel(BParams p) {
     const int gtid = blockIdx.x * NT + threadIdx.x, GT = gridDim.x * NT;
     const int gw = gtid >> 5, GW = GT >> 5;
     const int LS = p.LS;
-    __shared__ unsigned long long s_cnt[NT / 32][4];  // per-warp totals over completed batches
+    __shared__ unsigned long long s_cnt[NT / 32][5];  // per-warp totals over completed batches
     __shared__ int s_inexact;
     if (lane == 0)
-        for (int i = 0; i < 4; ++i) s_cnt[threadIdx.x >> 5][i] = 0ull;
+        for (int i = 0; i < 5; ++i) s_cnt[threadIdx.x >> 5][i] = 0ull;
     if (threadIdx.x == 0) s_inexact = 0;
     const long long nbatch = (p.k + BW - 1) / BW;
 
@@ -541,9 +543,9 @@ __global__ void __launch_bounds__(NT, 768 / NT) batch_kernel(BParams p) {
             }
         }
         if (!ovf) {  // overflowed batches are counted by the per-source rerun
-            unsigned long long v[4] = {cb.reached, cb.ar, cb.dag, cb.sc};
+            unsigned long long v[5] = {cb.reached, cb.ar, cb.dag, cb.sc, cb.dsum};
 #pragma unroll
-            for (int i = 0; i < 4; ++i) {
+            for (int i = 0; i < 5; ++i) {
 #pragma unroll
                 for (int o = 16; o > 0; o >>= 1) v[i] += __shfl_xor_sync(FULL, v[i], o);
                 if (lane == 0) s_cnt[threadIdx.x >> 5][i] += v[i];
@@ -561,6 +563,7 @@ __global__ void __launch_bounds__(NT, 768 / NT) batch_kernel(BParams p) {
         if (v[1]) atomicAdd(&p.stats->arcs_reached, v[1]);
         if (v[2]) atomicAdd(&p.stats->dag_arcs, v[2]);
         if (v[3]) atomicAdd(&p.stats->arcs_scanned, v[3]);
+        if (v[4]) atomicAdd(&p.stats->dist_sum, v[4]);
     }
     if (threadIdx.x == 0 && s_inexact) atomicOr(&p.stats->sigma_inexact, 1);
 }

@@ -202,6 +202,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             if (r == 0) {
                 if (tid == 0) {
                     ends[L + 1] = endL1;
+                    sm.st.dsum += (unsigned long long)L * (unsigned long long)tot;  // level L
                     lvl[(L + 2) & 3] = 0;  // next used for level L+2, reserved after barrier L+1
                 }
                 // hub words of level L's bitmap: every CTA read them before barrier L
@@ -302,6 +303,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             atomicAdd(&gs->levels, sm.st.lv[0]);
             atomicAdd(&gs->we_levels, sm.st.lv[0]);
             atomicAdd(&gs->n_reached, sm.st.reached);
+            atomicAdd(&gs->dist_sum, sm.st.dsum);
             atomicAdd(&gs->phase_cycles[0], sm.st.cyc[0]);
             atomicAdd(&gs->phase_cycles[2], sm.st.cyc[2]);
         }

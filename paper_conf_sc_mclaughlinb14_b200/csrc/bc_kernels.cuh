@@ -49,6 +49,7 @@ struct DevStats {
     int sampling_median;
     int pad;
     unsigned long long batches, batch_overflows;  // multi-source engine (bc_batch.cu)
+    unsigned long long dist_sum;  // sum over sources of sum_t d(s,t) over reached t (self-check)
 };
 
 struct KParams {
@@ -126,6 +127,7 @@ struct CtaStats {
     unsigned long long src, reached, ar, dg, sc;
     unsigned long long lv[2];   // levels expanded WE / EP
     unsigned long long cyc[4];  // fwd WE, fwd EP, bwd WE, bwd EP
+    unsigned long long dsum;    // sum of d(s,t) over the reached t of this CTA's sources
     int inexact;
 };
 
@@ -991,6 +993,7 @@ bc_kernel(KParams p) {
                 sm.st.cyc[mode] += (unsigned long long)dt;
                 if (p.dbg_fcyc && L < p.dbg_max_levels) p.dbg_fcyc[L] = dt;
                 sm.st.lv[mode] += 1;
+                sm.st.dsum += (unsigned long long)(L + 1) * (unsigned long long)(nhi - hi);
             }
             if (nhi == hi) break;  // Q_next_len == 0 (Alg. 2 l.11)
             mode = next_mode(p, mode, run_ep, hi - lo, nhi - hi);
@@ -1073,6 +1076,7 @@ bc_kernel(KParams p) {
         atomicAdd(&g->arcs_scanned, sm.st.sc);
 #pragma unroll
         for (int q = 0; q < 4; ++q) atomicAdd(&g->phase_cycles[q], sm.st.cyc[q]);
+        atomicAdd(&g->dist_sum, sm.st.dsum);
         if (sm.st.inexact) atomicOr(&g->sigma_inexact, 1);
     }
 }

@@ -59,6 +59,7 @@ int main(void){
   printf("%zu %zu %zu\n", offsetof(bc_stats, sampling_ep), offsetof(bc_stats, inflight),
          offsetof(bc_stats, kernel_ms));
   printf("%zu %zu %d\n", offsetof(bc_options, engine), offsetof(bc_options, group_ctas), BC_ENGINE_GROUP);
+  printf("%zu\n", offsetof(bc_stats, dist_sum));
   return 0; }
 """
     import tempfile
@@ -71,7 +72,7 @@ int main(void){
     O, S = _bc.bc_options, _bc.bc_stats
     assert vals == [ctypes.sizeof(O), O.gamma.offset, O.level_store.offset, ctypes.sizeof(S),
                     S.sampling_ep.offset, S.inflight.offset, S.kernel_ms.offset,
-                    O.engine.offset, O.group_ctas.offset, _bc.ENGINES["group"]]
+                    O.engine.offset, O.group_ctas.offset, _bc.ENGINES["group"], S.dist_sum.offset]
 
 
 def test_default_options_are_the_papers(lib):
@@ -79,6 +80,36 @@ def test_default_options_are_the_papers(lib):
     o = _bc.bc_default_options()
     assert (o.strategy, o.alpha, o.beta, o.gamma, o.n_samps, o.ep_min_frontier) == \
         (_bc.BC_STRATEGY_SAMPLING, 768, 512, 4.0, 512, 512)
+
+
+def test_default_options_overwrite_garbage(lib):
+    """A C caller's stack struct holds garbage: bc_default_options must set EVERY field
+    (round-1 bug: group_ctas was left as it was)."""
+    from paper_conf_sc_mclaughlinb14_b200 import _bc
+    o = _bc.bc_options()
+    ctypes.memset(ctypes.byref(o), 0xFF, ctypes.sizeof(o))
+    lib.bc_default_options(ctypes.byref(o))
+    z = _bc.bc_options()
+    lib.bc_default_options(ctypes.byref(z))          # from a zeroed struct
+    assert bytes(o) == bytes(z)
+    assert o.group_ctas == 0 and o.engine == _bc.BC_ENGINE_AUTO and o.hub_chunk == 0
+
+
+def test_pure_c_caller_compiles_and_links(lib, tmp_path):
+    """tests/c/abi_c1.c (a plain C program using only include/bc.h) links against libbc.so;
+    the GPU test test_gpu_abi_c.py runs it against the oracle."""
+    from paper_conf_sc_mclaughlinb14_b200 import _bc
+    exe = tmp_path / "abi_c1"
+    build_c_caller(str(exe))
+    out = subprocess.check_output(["ldd", str(exe)]).decode()
+    assert os.path.realpath(_bc.LIB_PATH) in out or "libbc.so" in out
+
+
+def build_c_caller(exe):
+    pkg = os.path.join(ROOT, "paper_conf_sc_mclaughlinb14_b200")
+    subprocess.check_call(["gcc", "-O2", "-std=c99", "-Wall", "-Werror", "-I", os.path.join(ROOT, "include"),
+                           "-o", exe, os.path.join(ROOT, "tests", "c", "abi_c1.c"),
+                           "-L", pkg, "-lbc", "-Wl,-rpath," + pkg, "-lm"])
 
 
 @pytest.mark.parametrize("case", ["ro0", "ron", "decreasing", "col_range", "neg_n", "big_nnz"])

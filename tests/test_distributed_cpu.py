@@ -58,3 +58,39 @@ def test_gloo_world2_equals_single_process(tmp_path, oracle_mod):
     whole = oracle_mod.bc(g, gg.sample_sources(g, 301, seed=2))
     assert np.array_equal(r0, r1)
     assert np.max(np.abs(r0 - whole) / np.maximum(np.abs(whole), 1)) < 1e-12
+
+
+def _worker_step(rank, world, port, out_dir, nsrc):
+    """Drives distributed.bc_step -- the function bench.py times -- with a CPU compute;
+    nsrc < world leaves some ranks with an EMPTY shard (their partial BC must be zero,
+    not "all vertices")."""
+    import torch
+    import torch.distributed as dist
+    import oracle
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import bench
+    cfg, g, total, local = bench.make_workload("c1", world, rank, "strong", nsrc)
+    out = torch.empty(g.n, dtype=torch.float64)
+    bdist.bc_step(lambda o: o.copy_(torch.from_numpy(oracle.bc(g, local))), out)
+    np.save(os.path.join(out_dir, f"s{rank}.npy"), out.numpy())
+    np.save(os.path.join(out_dir, f"src{rank}.npy"), local)
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,nsrc", [(2, 301), (3, 2)])
+def test_gloo_bench_step(tmp_path, oracle_mod, world, nsrc):
+    port = _free_port()
+    mp.spawn(_worker_step, args=(world, port, str(tmp_path), nsrc), nprocs=world, join=True)
+    outs = [np.load(tmp_path / f"s{r}.npy") for r in range(world)]
+    shards = [np.load(tmp_path / f"src{r}.npy") for r in range(world)]
+    g = gg.CONFIGS["c1"].graph()
+    total = gg.sample_sources(g, nsrc, gg.CONFIGS["c1"].seed + 7)
+    assert sorted(np.concatenate(shards).tolist()) == sorted(total.tolist())
+    if nsrc < world:
+        assert min(s.size for s in shards) == 0
+    whole = oracle_mod.bc(g, total)
+    for o in outs:
+        assert np.array_equal(o, outs[0])
+        assert np.max(np.abs(o - whole) / np.maximum(np.abs(whole), 1)) < 1e-12

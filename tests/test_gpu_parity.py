@@ -450,3 +450,28 @@ def test_fig1_consistent_golden(bcmod, oracle_mod, strategy):
         for s in range(g.n):
             check_source(bg, g, s, oracle_mod)
         assert rel_err(bg.compute(None), want) < 1e-12
+
+
+def test_compute_device_empty_source_tensor(bcmod):
+    """An empty CUDA tensor has data_ptr() == 0; it must mean "no sources" (BC = 0), not
+    the C ABI's NULL = "all vertices" (an empty multi-GPU shard)."""
+    import torch
+    g = graph("c1")
+    with bcmod.BCGraph.from_graph(g) as bg:
+        out = torch.full((g.n,), 3.0, dtype=torch.float64, device="cuda")
+        bg.compute_device(torch.zeros(0, dtype=torch.int32, device="cuda"), out)
+        torch.cuda.synchronize()
+        assert float(out.abs().max()) == 0.0
+        assert bg.stats()["sources"] == 0
+
+
+def test_seq_max_deg_shrink_reallocates_bigq(bcmod, oracle_mod):
+    """lowering the effective row-split threshold (seq_max_deg) must grow the
+    hub-row queue (bigq); c4's hubs then all go to the CTA-cooperative phase."""
+    g = graph("c4")
+    src = gg.CONFIGS["c4"].sources(g)[:40]
+    with bcmod.BCGraph.from_graph(g, strategy="we", seq_max_deg=20000, inflight=7) as bg:
+        bg.set_options(seq_max_deg=0)   # effective threshold 20000 -> 8192: bigq must grow
+        check_bc(bg, g, src, oracle_mod)
+        bg.set_options(seq_max_deg=4, warp_max_deg=8)
+        check_bc(bg, g, src, oracle_mod)
