@@ -6,7 +6,7 @@ ARCH := -gencode arch=compute_100a,code=sm_100a
 NVFLAGS := -O3 -std=c++17 -lineinfo $(ARCH) -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
            -Iinclude -Xptxas -v
 CSRC := $(PKG)/csrc
-HDRS := $(CSRC)/bc_kernels.cuh $(CSRC)/bc_batch.cuh $(CSRC)/bc_group.cuh include/bc.h
+HDRS := $(CSRC)/bc_kernels.cuh $(CSRC)/bc_fast.cuh $(CSRC)/bc_batch.cuh $(CSRC)/bc_group.cuh include/bc.h
 # one translation unit per level store (compiled in parallel: make -j)
 UNITS := bc_api bc_batch bc_group bc_inst_directed bc_inst_levels bc_inst_gcodes bc_inst_scodes
 OBJS := $(UNITS:%=build/%.o)

@@ -103,6 +103,7 @@ struct bc_graph {
         int nt = 256;
         size_t dyn = 0;   // dynamic shared memory bytes
         int per_sm = 1;   // resident CTAs per SM
+        int smem_nb = 0;  // fast path: the discovery bitmap is in dynamic smem after the codes
     } cfg_we, cfg_ep;
     int lstore = 1;       // level store: 1 int32 d (HBM), 2 codes in SMEM, 3 codes in HBM/L2
     uint32_t *gcodes = nullptr, *gfb = nullptr;
@@ -318,6 +319,7 @@ static int configure(bc_graph *g) {
     g->cfg_we.nt = g->cfg_ep.nt = nt;
     g->cfg_we.dyn = g->lstore == 2 ? code_bytes : 0;
     g->cfg_ep.dyn = g->lstore == 2 ? code_bytes + fb_bytes : 0;
+    g->cfg_we.smem_nb = g->cfg_ep.smem_nb = 0;
     CK(cudaFuncSetAttribute(g->cfg_we.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_we.dyn));
     CK(cudaFuncSetAttribute(g->cfg_ep.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_ep.dyn));
     for (auto *c : {&g->cfg_we, &g->cfg_ep}) {
@@ -325,6 +327,26 @@ static int configure(bc_graph *g) {
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, c->fn, c->nt, c->dyn));
         if (per_sm < 1) return fail(BC_EINTERNAL, "kernel cannot be resident (dyn smem %zu)", c->dyn);
         c->per_sm = per_sm;
+    }
+    // Fast path (bc_fast.cuh: undirected, shared-memory codes, WE-only kernel without the
+    // successor bitmap): the sorted-frontier discovery bitmap goes to shared memory too,
+    // after the codes, when that costs no resident CTA.
+    if (g->lstore == 2 && !g->directed && !g->succ_bits && g->sort_frontier) {
+        bc_graph::KCfg &c = g->cfg_we;
+        const size_t dyn2 = code_bytes + 4 * (size_t)g->nb_words;
+        int max_optin = 0;
+        CK(cudaDeviceGetAttribute(&max_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, g->device));
+        if (dyn2 + 16 * 1024 <= (size_t)max_optin) {
+            CK(cudaFuncSetAttribute(c.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn2));
+            int per_sm = 0;
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, c.fn, c.nt, dyn2));
+            if (per_sm >= c.per_sm) {
+                c.dyn = dyn2;
+                c.smem_nb = 1;
+            } else {
+                CK(cudaFuncSetAttribute(c.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.dyn));
+            }
+        }
     }
     return BC_OK;
 }
@@ -767,6 +789,9 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col_in) 
     g->graph_bytes = b_ro + 2 * b_col;
     CK(cudaMemcpy(g->ro, ro32.data(), sizeof(int) * ((size_t)n + 1), cudaMemcpyHostToDevice));
     if (nnz) CK(cudaMemcpy(g->col, col, sizeof(int) * (size_t)nnz, cudaMemcpyHostToDevice));
+    // zeroed slack after the last column: 16-byte quad reads past a row's end (one-thread
+    // rows) then always see valid vertex ids
+    CK(cudaMemset(g->col + nnz, 0, 16));
     if (nnz && n) {
         build_src_kernel<<<std::min((nnz + 255) / 256, 148 * 16), 256>>>(g->ro, n, nnz, g->src);
         CK(cudaGetLastError());
@@ -947,11 +972,23 @@ static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
     // (Alg. 4) vertices; when no frontier can be that large, the work-efficient-only
     // kernel (no EP code, no bitmap) is launched instead.
     const bool ep_possible =
-        p.launch_mode == LM_EP ||
-        (p.launch_mode == LM_SAMPLED && (long long)p.ep_min_frontier <= (long long)g->n) ||
-        (p.launch_mode == LM_HYBRID && (long long)p.beta < (long long)g->n);
+        !p.skip_if_ep &&
+        (p.launch_mode == LM_EP ||
+         (p.launch_mode == LM_SAMPLED && (long long)p.ep_min_frontier <= (long long)g->n) ||
+         (p.launch_mode == LM_HYBRID && (long long)p.beta < (long long)g->n));
+    // Alg. 5 run whose decision is still on the device: enqueue BOTH kernels, each gated on
+    // the flag (the other exits at once), so a WE decision runs the WE-only kernel and never
+    // pays for the EP code path (the selectors taxed WE levels 2x).
+    if (ep_possible && p.launch_mode == LM_SAMPLED && p.sampled_flag && !p.skip_if_we) {
+        KParams pw = p;
+        pw.skip_if_ep = 1;
+        int rc = launch(g, pw, st);
+        if (rc) return rc;
+        p.skip_if_we = 1;
+    }
     const bc_graph::KCfg &c = ep_possible ? g->cfg_ep : g->cfg_we;
     p.fb_words = ep_possible ? g->fb_words : 0;
+    p.smem_nb = c.smem_nb;
     const long long cap = std::min<long long>(g->slots, (long long)c.per_sm * g->num_sms);
     const int grid = (int)std::min<long long>(cap, p.k);
     void *args[] = {&p};

@@ -1,0 +1,290 @@
+// bc_fast.cuh -- the work-efficient fast path of bc_kernel for undirected graphs whose 2-bit
+// level codes live in shared memory (bc_kernel<false, SmemCodes, NT, false, false>: every
+// Alg. 5 run with the B200 guard and every WE run on n <= ~2^18, i.e. c1..c4).
+//
+// Same arithmetic, same order and same outputs as the generic row_pass / forward_we /
+// backward_we (Alg. 2 l.3-8 as a pull; Alg. 3 l.5-9; Eq. 3),
+// written for fewer issued instructions per arc (ncu r01: 2.07 warp instructions and ~56
+// thread instructions per scanned arc, issue-bound at 61 %):
+//  * the probe of a 2-bit code is one LDS + one funnel rotate (the rotate amount 2u mod 32
+//    is taken from u << 1 by the hardware's mod-32 wrap) + one AND;
+//  * sigma / omega gathers are PREDICATED loads (no select, no branch);
+//  * one-thread rows run a warp-uniform quad loop (trip count = the chunk's longest row),
+//    so claims are gated by one warp vote per quad and issued as predicated shared atomics;
+//  * large levels discover into a shared-memory bitmap only (no S append: the level is
+//    rebuilt in vertex order from the bitmap anyway), small levels append to S with one
+//    shared atomic per warp and arc slot;
+//  * DAG arcs are counted from a per-quad predicate mask (one POPC), not per arc.
+// One-thread rows still sum in CSR order (= the oracle's order, DESIGN R4).
+#pragma once
+
+namespace bcdev {
+
+__device__ __forceinline__ int code_at(const uint32_t *sw, int u) {
+    const uint32_t wd = sw[(unsigned)u >> 4];
+    return (int)(__funnelshift_r(wd, wd, (unsigned)u << 1) & 3u);  // rotate by 2(u mod 16)
+}
+
+// v = c ? *p : 0.0, as a predicated ld.global.ca (L1-cached; see ld_sig).
+__device__ __forceinline__ double ldca_if(const double *p, bool c) {
+    double v;
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\tmov.f64 %0, 0d0000000000000000;\n\t"
+        "@q ld.global.ca.f64 %0, [%1];\n\t}"
+        : "=d"(v)
+        : "l"(p), "r"((unsigned)c));
+    return v;
+}
+
+// old word if c (atomic OR into shared memory), else 0.
+__device__ __forceinline__ uint32_t atom_or_shared_if(uint32_t *addr, uint32_t val, bool c) {
+    uint32_t old = 0u;
+    const unsigned a = (unsigned)__cvta_generic_to_shared(addr);
+    asm volatile(
+        "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\t@q atom.shared.or.b32 %0, [%1], %2;\n\t}"
+        : "+r"(old)
+        : "r"(a), "r"(val), "r"((unsigned)c)
+        : "memory");
+    return old;
+}
+
+__device__ __forceinline__ void red_or_shared_if(uint32_t *addr, uint32_t val, bool c) {
+    const unsigned a = (unsigned)__cvta_generic_to_shared(addr);
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.or.b32 [%0], %1;\n\t}"
+                 :
+                 : "r"(a), "r"(val), "r"((unsigned)c)
+                 : "memory");
+}
+
+// Per-level context of the fast path.
+struct FastLevel {
+    uint32_t *sw;      // shared 2-bit codes
+    uint32_t *snb;     // shared discovery bitmap of level L+1 (nullptr: append to S)
+    uint32_t *gnb;     // queue mode: also mark winners in this global bitmap (sorted frontiers
+                       // of EP-capable kernels, rebuilt by the kernel when the level is large)
+    double *sig;       // sigma (forward) / sigma-then-omega (backward), this slot
+    int *Snext;        // S + hi: where level L+1 is appended (queue mode)
+    int *cnt;          // &sm.cnt[L % 3]
+    int kmatch;        // forward: key(L-1) (predecessors); backward: key(L+1) (successors)
+    int knew;          // forward: key(L+1), the code a discovery sets (as a 2-bit value)
+};
+
+// Claims of up to four neighbours (forward only): predicated shared atomics on the code
+// words, winners recorded in the bitmap or appended to S.  Warp-uniform call.
+__device__ __forceinline__ void fast_claims(const FastLevel &f, const int (&u)[4], const bool (&un)[4]) {
+    bool won[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const unsigned sh = ((unsigned)u[j] << 1) & 30u;
+        const uint32_t old = atom_or_shared_if(&f.sw[(unsigned)u[j] >> 4], (uint32_t)f.knew << sh, un[j]);
+        won[j] = un[j] && ((old >> sh) & 3u) == 0u;
+    }
+    if (f.snb) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) red_or_shared_if(&f.snb[(unsigned)u[j] >> 5], 1u << (u[j] & 31), won[j]);
+    } else {
+        const int lane = threadIdx.x & 31;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const unsigned m = __ballot_sync(FULL, won[j]);
+            if (m) {
+                int base = 0;
+                if (lane == __ffs(m) - 1) base = atomicAdd(f.cnt, __popc(m));
+                base = __shfl_sync(FULL, base, __ffs(m) - 1);
+                if (won[j]) {
+                    f.Snext[base + __popc(m & ((1u << lane) - 1u))] = u[j];
+                    if (f.gnb) atomicOr(&f.gnb[(unsigned)u[j] >> 5], 1u << (u[j] & 31));  // RED
+                }
+            }
+        }
+    }
+}
+
+// Quads of the one-thread rows of a 32-vertex chunk; lane = row [beg, end) (deg <= seq_max,
+// deg = 0 for lanes without a row).  Warp-uniform trip count.  Returns the lane's sum of
+// gathers in CSR order.
+template <bool FWD>
+__device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *__restrict__ cols, int beg,
+                                                int end, Counters &c) {
+    const int q0 = beg & ~3;
+    const int nq = end > beg ? ((end + 3) >> 2) - (beg >> 2) : 0;
+    const int maxq = __reduce_max_sync(FULL, (unsigned)nq);
+    double acc = 0.0;
+    int4 nx = make_int4(0, 0, 0, 0);
+    if (nq > 0) nx = *reinterpret_cast<const int4 *>(cols + q0);
+    unsigned dag = 0;
+    for (int q = 0; q < maxq; ++q) {
+        const int pos = q0 + 4 * q;
+        const int4 c4 = nx;
+        if (q + 1 < nq) nx = *reinterpret_cast<const int4 *>(cols + pos + 4);
+        unsigned valid = q < nq ? 0xFu : 0u;
+        if (pos < beg) valid &= 0xFu << (beg - pos);
+        if (pos + 4 > end) valid &= 0xFu >> min(4, pos + 4 - end);
+        // slots outside the row hold other rows' columns (or the zeroed slack after col[nnz-1]):
+        // valid vertex ids, probed harmlessly and masked out of every predicate
+        const int u[4] = {c4.x, c4.y, c4.z, c4.w};
+        int k[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) k[j] = code_at(f.sw, u[j]);
+        bool pg[4];
+        double g[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            pg[j] = ((valid >> j) & 1u) && k[j] == f.kmatch;
+            g[j] = ldca_if(f.sig + u[j], pg[j]);
+        }
+        if (FWD) {
+            bool un[4];
+            bool any = false;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                un[j] = ((valid >> j) & 1u) && k[j] == 0;
+                any |= un[j];
+            }
+            if (__any_sync(FULL, any)) fast_claims(f, u, un);
+            dag += (unsigned)pg[0] + (unsigned)pg[1] + (unsigned)pg[2] + (unsigned)pg[3];
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc += g[j];
+    }
+    if (FWD) c.dag += dag;
+    return acc;
+}
+
+// One row [b, e) expanded by `stride` cooperating threads (a warp or the CTA), thread t
+// taking arcs t, t + stride, ... (four in flight).  Warp-uniform within each warp.  Returns
+// the thread's partial sum (the caller reduces).
+template <bool FWD>
+__device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *__restrict__ cols, int b, int e,
+                                                int t, int stride, Counters &c) {
+    double acc = 0.0;
+    unsigned dag = 0;
+    int un_[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) un_[j] = b + t + j * stride < e ? cols[b + t + j * stride] : 0;
+    for (int base = b; base < e; base += 4 * stride) {
+        int u[4];
+        bool ok[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            u[j] = un_[j];
+            ok[j] = base + t + j * stride < e;
+        }
+        const int bn = base + 4 * stride;
+        if (bn < e) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j) un_[j] = bn + t + j * stride < e ? cols[bn + t + j * stride] : 0;
+        }
+        int k[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) k[j] = code_at(f.sw, u[j]);
+        bool pg[4];
+        double g[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            pg[j] = ok[j] && k[j] == f.kmatch;
+            g[j] = ldca_if(f.sig + u[j], pg[j]);
+        }
+        if (FWD) {
+            bool un[4];
+            bool any = false;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                un[j] = ok[j] && k[j] == 0;
+                any |= un[j];
+            }
+            if (__any_sync(FULL, any)) fast_claims(f, u, un);
+            dag += (unsigned)pg[0] + (unsigned)pg[1] + (unsigned)pg[2] + (unsigned)pg[3];
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc += g[j];
+    }
+    if (FWD) c.dag += dag;
+    return acc;
+}
+
+// One forward (FWD) or backward level over S[lo, hi): phase A (warps take 32-vertex chunks:
+// one-thread rows, then warp rows one at a time), phase B (rows > warp_max, whole CTA).
+// Forward finish: sigma[v] = sum (L > 0).  Backward finish: finish_dependency (omega in
+// place, bc += delta).  Ends with a CTA barrier (in phase B's test).
+template <int NT, bool FWD>
+__device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, const int *__restrict__ S, int lo,
+                                          int hi, int L, int *bigq, Smem<NT> &sm, Counters &c) {
+    constexpr int NW = NT / 32;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int *__restrict__ rows = p.ro;
+    const int *__restrict__ cols = p.col;
+    const int seq_max = p.seq_max_deg, warp_max = p.warp_max_deg;
+    for (int base = lo + wid * 32; base < hi; base += NT) {
+        const int i = base + lane;
+        int v = -1, beg = 0, deg = 0;
+        if (i < hi) {
+            v = S[i];
+            beg = rows[v];
+            deg = rows[v + 1] - beg;
+        }
+        c.scanned += deg;
+        const bool seq = v >= 0 && deg <= seq_max;
+        double sw = 0.0;
+        if (!FWD && seq) sw = __ldcg(&f.sig[v]);  // sigma[w], issued early
+        const double acc = fast_seq_rows<FWD>(f, cols, beg, seq ? beg + deg : beg, c);
+        if (seq) {
+            if (FWD) {
+                if (L > 0) f.sig[v] = acc;
+            } else {
+                finish_dependency(p, sw, f.sig, v, acc);
+            }
+        }
+        unsigned med = __ballot_sync(FULL, v >= 0 && deg > seq_max && deg <= warp_max);
+        while (med) {
+            const int leader = __ffs(med) - 1;
+            med &= med - 1;
+            const int w = __shfl_sync(FULL, v, leader);
+            const int b = __shfl_sync(FULL, beg, leader);
+            const int e = b + __shfl_sync(FULL, deg, leader);
+            double swm = 0.0;
+            if (!FWD && lane == leader) swm = __ldcg(&f.sig[w]);
+            const double a = warp_sum(fast_coop_row<FWD>(f, cols, b, e, lane, 32, c));
+            if (lane == leader) {
+                if (FWD) {
+                    if (L > 0) {
+                        f.sig[w] = a;
+                        if (a >= TWO53) c.inexact = 1;
+                    }
+                } else {
+                    finish_dependency(p, swm, f.sig, w, a);
+                }
+            }
+        }
+        if (v >= 0 && deg > warp_max) bigq[atomicAdd(&sm.nbig, 1)] = v;
+    }
+    if (__syncthreads_or(sm.nbig > 0)) {
+        const int nb = sm.nbig;
+        for (int r = 0; r < nb; ++r) {
+            const int v = __ldcg(&bigq[r]);
+            const int b = rows[v], e = rows[v + 1];
+            double swb = 0.0;
+            if (!FWD && threadIdx.x == 0) swb = __ldcg(&f.sig[v]);
+            const double a = warp_sum(fast_coop_row<FWD>(f, cols, b, e, threadIdx.x, NT, c));
+            if (lane == 0) sm.red[wid] = a;
+            __syncthreads();
+            if (threadIdx.x == 0) {
+                double t = 0.0;
+#pragma unroll
+                for (int q = 0; q < NW; ++q) t += sm.red[q];
+                if (FWD) {
+                    if (L > 0) {
+                        f.sig[v] = t;
+                        if (t >= TWO53) c.inexact = 1;
+                    }
+                } else {
+                    finish_dependency(p, swb, f.sig, v, t);
+                }
+                if (r == nb - 1) sm.nbig = 0;
+            }
+            __syncthreads();
+        }
+    }
+}
+
+}  // namespace bcdev
