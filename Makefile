@@ -11,7 +11,7 @@ HDRS := $(CSRC)/bc_kernels.cuh $(CSRC)/bc_fast.cuh $(CSRC)/bc_batch.cuh $(CSRC)/
 UNITS := bc_api bc_batch bc_group bc_inst_directed bc_inst_levels bc_inst_gcodes bc_inst_scodes
 OBJS := $(UNITS:%=build/%.o)
 
-all: $(PKG)/libbc.so $(PKG)/libgraphgen.so oracle/liboracle.so
+all: $(PKG)/libbc.so $(PKG)/libgraphgen.so $(PKG)/libbcprobe.so oracle/liboracle.so
 
 build/%.o: $(CSRC)/%.cu $(HDRS)
 	@mkdir -p build
@@ -22,6 +22,10 @@ $(PKG)/libbc.so: $(OBJS)
 	@cat $(UNITS:%=build/%.ptxas.log) > $(CSRC)/ptxas.log
 	@grep -E "registers|spill" $(CSRC)/ptxas.log | sed 's/^ptxas info    : //' | sort -u | head -20
 
+# measurement helper for bench.py (L2 read ceiling), not part of the method
+$(PKG)/libbcprobe.so: $(CSRC)/l2probe.cu
+	$(NVCC) -O3 -std=c++17 $(ARCH) -Xcompiler -fPIC -Xcompiler -fvisibility=hidden -shared -o $@ $<
+
 $(PKG)/libgraphgen.so: $(PKG)/graphgen_native.c
 	gcc -O2 -std=c99 -fPIC -shared -pthread -o $@ $<
 
@@ -29,7 +33,7 @@ oracle/liboracle.so: oracle/brandes_oracle.c
 	gcc -O2 -std=c99 -fPIC -shared -pthread -o $@ $<
 
 clean:
-	rm -rf build $(PKG)/libbc.so $(PKG)/libgraphgen.so oracle/liboracle.so
+	rm -rf build $(PKG)/libbc.so $(PKG)/libgraphgen.so $(PKG)/libbcprobe.so oracle/liboracle.so
 
 .PHONY: all clean
 

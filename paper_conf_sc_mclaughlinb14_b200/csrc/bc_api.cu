@@ -103,13 +103,12 @@ struct bc_graph {
         int nt = 256;
         size_t dyn = 0;   // dynamic shared memory bytes
         int per_sm = 1;   // resident CTAs per SM
-        int smem_nb = 0;  // fast path: the discovery bitmap is in dynamic smem after the codes
     } cfg_we, cfg_ep;
     int lstore = 1;       // level store: 1 int32 d (HBM), 2 codes in SMEM, 3 codes in HBM/L2
     uint32_t *gcodes = nullptr, *gfb = nullptr;
     int sort_frontier = 0, sort_min = 0, nb_words = 0;  // sorted-frontier rebuild (configure())
     uint32_t *nbits = nullptr;
-    int succ_bits = 0, sb_words = 0;                    // successor bitmap over arcs
+    int succ_bits = 0, sb_words = 0;                    // successor bitmap over arcs (generic kernels)
     uint32_t *sbits = nullptr;
     int code_words = 0, fb_words = 0;
     int seq_max_deg = 32;
@@ -319,7 +318,6 @@ static int configure(bc_graph *g) {
     g->cfg_we.nt = g->cfg_ep.nt = nt;
     g->cfg_we.dyn = g->lstore == 2 ? code_bytes : 0;
     g->cfg_ep.dyn = g->lstore == 2 ? code_bytes + fb_bytes : 0;
-    g->cfg_we.smem_nb = g->cfg_ep.smem_nb = 0;
     CK(cudaFuncSetAttribute(g->cfg_we.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_we.dyn));
     CK(cudaFuncSetAttribute(g->cfg_ep.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)g->cfg_ep.dyn));
     for (auto *c : {&g->cfg_we, &g->cfg_ep}) {
@@ -327,26 +325,6 @@ static int configure(bc_graph *g) {
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, c->fn, c->nt, c->dyn));
         if (per_sm < 1) return fail(BC_EINTERNAL, "kernel cannot be resident (dyn smem %zu)", c->dyn);
         c->per_sm = per_sm;
-    }
-    // Fast path (bc_fast.cuh: undirected, shared-memory codes, WE-only kernel without the
-    // successor bitmap): the sorted-frontier discovery bitmap goes to shared memory too,
-    // after the codes, when that costs no resident CTA.
-    if (g->lstore == 2 && !g->directed && !g->succ_bits && g->sort_frontier) {
-        bc_graph::KCfg &c = g->cfg_we;
-        const size_t dyn2 = code_bytes + 4 * (size_t)g->nb_words;
-        int max_optin = 0;
-        CK(cudaDeviceGetAttribute(&max_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, g->device));
-        if (dyn2 + 16 * 1024 <= (size_t)max_optin) {
-            CK(cudaFuncSetAttribute(c.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn2));
-            int per_sm = 0;
-            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, c.fn, c.nt, dyn2));
-            if (per_sm >= c.per_sm) {
-                c.dyn = dyn2;
-                c.smem_nb = 1;
-            } else {
-                CK(cudaFuncSetAttribute(c.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)c.dyn));
-            }
-        }
     }
     return BC_OK;
 }
@@ -988,7 +966,6 @@ static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
     }
     const bc_graph::KCfg &c = ep_possible ? g->cfg_ep : g->cfg_we;
     p.fb_words = ep_possible ? g->fb_words : 0;
-    p.smem_nb = c.smem_nb;
     const long long cap = std::min<long long>(g->slots, (long long)c.per_sm * g->num_sms);
     const int grid = (int)std::min<long long>(cap, p.k);
     void *args[] = {&p};

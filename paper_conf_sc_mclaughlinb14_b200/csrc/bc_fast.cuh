@@ -10,11 +10,11 @@
 //    is taken from u << 1 by the hardware's mod-32 wrap) + one AND;
 //  * sigma / omega gathers are PREDICATED loads (no select, no branch);
 //  * one-thread rows run a warp-uniform quad loop (trip count = the chunk's longest row),
-//    so claims are gated by one warp vote per quad and issued as predicated shared atomics;
-//  * large levels discover into a shared-memory bitmap only (no S append: the level is
-//    rebuilt in vertex order from the bitmap anyway), small levels append to S with one
-//    shared atomic per warp and arc slot;
-//  * DAG arcs are counted from a per-quad predicate mask (one POPC), not per arc.
+//    so claims are gated by one warp vote per quad and issued as predicated shared atomics
+//    (a per-lane trip count with per-slot claims was measured 4 % slower on c4);
+//  * discoveries are appended to S with one shared atomic per warp and arc slot (and marked
+//    in the sorted-frontier bitmap when the level is likely to be large);
+//  * DAG arcs are counted per quad from the gather predicates.
 // One-thread rows still sum in CSR order (= the oracle's order, DESIGN R4).
 #pragma once
 
@@ -48,20 +48,11 @@ __device__ __forceinline__ uint32_t atom_or_shared_if(uint32_t *addr, uint32_t v
     return old;
 }
 
-__device__ __forceinline__ void red_or_shared_if(uint32_t *addr, uint32_t val, bool c) {
-    const unsigned a = (unsigned)__cvta_generic_to_shared(addr);
-    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.shared.or.b32 [%0], %1;\n\t}"
-                 :
-                 : "r"(a), "r"(val), "r"((unsigned)c)
-                 : "memory");
-}
-
 // Per-level context of the fast path.
 struct FastLevel {
     uint32_t *sw;      // shared 2-bit codes
-    uint32_t *snb;     // shared discovery bitmap of level L+1 (nullptr: append to S)
-    uint32_t *gnb;     // queue mode: also mark winners in this global bitmap (sorted frontiers
-                       // of EP-capable kernels, rebuilt by the kernel when the level is large)
+    uint32_t *gnb;     // non-null: discoveries go to this level bitmap ONLY (no S append); the
+                       // kernel rebuilds level L+1 from it in vertex order (sorted frontiers)
     double *sig;       // sigma (forward) / sigma-then-omega (backward), this slot
     int *Snext;        // S + hi: where level L+1 is appended (queue mode)
     int *cnt;          // &sm.cnt[L % 3]
@@ -69,8 +60,17 @@ struct FastLevel {
     int knew;          // forward: key(L+1), the code a discovery sets (as a 2-bit value)
 };
 
+__device__ __forceinline__ void red_or_global_if(uint32_t *addr, uint32_t val, bool c) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.global.or.b32 [%0], %1;\n\t}"
+                 :
+                 : "l"(addr), "r"(val), "r"((unsigned)c)
+                 : "memory");
+}
+
 // Claims of up to four neighbours (forward only): predicated shared atomics on the code
-// words, winners recorded in the bitmap or appended to S.  Warp-uniform call.
+// words; winners are marked in the level bitmap (large levels: the kernel rebuilds level
+// L+1 from it in vertex order) or appended to S with ONE warp scan and ONE shared atomic
+// for all four slots.  Warp-uniform call.
 __device__ __forceinline__ void fast_claims(const FastLevel &f, const int (&u)[4], const bool (&un)[4]) {
     bool won[4];
 #pragma unroll
@@ -79,25 +79,27 @@ __device__ __forceinline__ void fast_claims(const FastLevel &f, const int (&u)[4
         const uint32_t old = atom_or_shared_if(&f.sw[(unsigned)u[j] >> 4], (uint32_t)f.knew << sh, un[j]);
         won[j] = un[j] && ((old >> sh) & 3u) == 0u;
     }
-    if (f.snb) {
+    if (f.gnb) {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) red_or_shared_if(&f.snb[(unsigned)u[j] >> 5], 1u << (u[j] & 31), won[j]);
-    } else {
-        const int lane = threadIdx.x & 31;
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            const unsigned m = __ballot_sync(FULL, won[j]);
-            if (m) {
-                int base = 0;
-                if (lane == __ffs(m) - 1) base = atomicAdd(f.cnt, __popc(m));
-                base = __shfl_sync(FULL, base, __ffs(m) - 1);
-                if (won[j]) {
-                    f.Snext[base + __popc(m & ((1u << lane) - 1u))] = u[j];
-                    if (f.gnb) atomicOr(&f.gnb[(unsigned)u[j] >> 5], 1u << (u[j] & 31));  // RED
-                }
-            }
-        }
+        for (int j = 0; j < 4; ++j) red_or_global_if(&f.gnb[(unsigned)u[j] >> 5], 1u << (u[j] & 31), won[j]);
+        return;
     }
+    const int lane = threadIdx.x & 31;
+    const int cnt = (int)won[0] + (int)won[1] + (int)won[2] + (int)won[3];
+    int incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+    }
+    const int tot = __shfl_sync(FULL, incl, 31);
+    if (tot == 0) return;
+    int base = 0;
+    if (lane == 31) base = atomicAdd(f.cnt, tot);
+    base = __shfl_sync(FULL, base, 31) + incl - cnt;
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+        if (won[j]) f.Snext[base++] = u[j];
 }
 
 // Quads of the one-thread rows of a 32-vertex chunk; lane = row [beg, end) (deg <= seq_max,
@@ -154,6 +156,10 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
 // One row [b, e) expanded by `stride` cooperating threads (a warp or the CTA), thread t
 // taking arcs t, t + stride, ... (four in flight).  Warp-uniform within each warp.  Returns
 // the thread's partial sum (the caller reduces).
+//
+// (Successor bits for these rows -- forward ballots + REDs marking the DAG arcs, backward
+// visiting only marked arcs -- were measured slower on B200: c4 161 -> 188 ms per 4,096
+// sources, the forward paying more than the backward saved.)
 template <bool FWD>
 __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *__restrict__ cols, int b, int e,
                                                 int t, int stride, Counters &c) {

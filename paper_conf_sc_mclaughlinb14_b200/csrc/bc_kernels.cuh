@@ -92,7 +92,6 @@ struct KParams {
     size_t stride_nb;
     int nb_words;
     int sort_min;        // rebuild a level in vertex order when it has >= sort_min vertices
-    int smem_nb;         // fast path: the discovery bitmap follows the codes in dynamic smem
     uint32_t *sbits;     // per-slot successor bitmap over arcs (ArcBits), NULL = off
     size_t stride_sb;
     int sb_words;        // multiple of 4
@@ -616,14 +615,14 @@ __device__ __forceinline__ int next_mode(const KParams &p, int mode, int run_ep,
 // Rewrite out[0 .. popcount(nb)) with the set bits of nb in ascending order and
 // clear nb.  Each warp owns a contiguous range of words and reads it coalesced;
 // one block scan of the warp totals.  Returns popcount(nb); ends with a barrier.
-template <int NT, bool SHARED = false>
+template <int NT>
 __device__ __forceinline__ int compact_level(uint32_t *nb, int words, int *out, Smem<NT> &sm) {
     constexpr int NW = NT / 32;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int per = ((words + NW - 1) / NW + 31) & ~31;  // words per warp, multiple of 32
     const int w0 = min(wid * per, words), w1 = min(w0 + per, words);
     int cnt = 0;
-    for (int w = w0 + lane; w < w1; w += 32) cnt += __popc(SHARED ? nb[w] : __ldcg(&nb[w]));
+    for (int w = w0 + lane; w < w1; w += 32) cnt += __popc(__ldcg(&nb[w]));
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
     if (lane == 0) sm.wtot[wid] = cnt;
@@ -635,7 +634,7 @@ __device__ __forceinline__ int compact_level(uint32_t *nb, int words, int *out, 
     }
     for (int w = w0; w < w1; w += 32) {
         const int wi = w + lane;
-        uint32_t bits = wi < w1 ? (SHARED ? nb[wi] : __ldcg(&nb[wi])) : 0u;
+        uint32_t bits = wi < w1 ? __ldcg(&nb[wi]) : 0u;
         const int c = __popc(bits);
         int incl = c;
 #pragma unroll
@@ -931,13 +930,14 @@ bc_kernel(KParams p) {
     int *bigq = p.bigq + slot * p.stride_big;
     uint32_t *nb = p.nbits ? p.nbits + slot * p.stride_nb : nullptr;
     uint32_t *sb = SB && p.sbits ? p.sbits + slot * p.stride_sb : nullptr;
-    // Fast path (bc_fast.cuh) for the work-efficient levels of undirected graphs with
-    // shared-memory codes; WE-only kernels also keep the discovery bitmap in shared memory.
-    constexpr bool FASTWE = !DIR && !SB && std::is_same<LV, SmemCodes>::value;
-    constexpr bool FAST = FASTWE && !EPOK;
-    uint32_t *const snb = (FAST && p.smem_nb) ? dyn_smem + p.code_words : nullptr;
-    if (snb)
-        for (int i = threadIdx.x; i < p.nb_words; i += NT) snb[i] = 0u;
+    // Fast path (bc_fast.cuh): undirected graphs, shared-memory codes, WE-only kernels.
+    // (Also running the EP-capable kernels' WE levels through it was measured slower on B200:
+    // c4 hybrid 234 -> 348 ms.)
+#ifdef BC_NO_FAST
+    constexpr bool FAST = false;
+#else
+    constexpr bool FAST = !DIR && !SB && !EPOK && std::is_same<LV, SmemCodes>::value;
+#endif
 
     Counters c;
     const int run_ep = (p.launch_mode == LM_SAMPLED && p.sampled_flag) ? *p.sampled_flag : 0;
@@ -981,13 +981,10 @@ bc_kernel(KParams p) {
             uint32_t *const nbl =
                 LV::BITMAP_DISCOVERY ? nb
                                      : ((nb && (long long)(hi - lo) * 4 >= p.sort_min) ? nb : nullptr);
-            // fast path: a level likely to be large discovers into the shared bitmap only
-            uint32_t *const fnb = (snb && (long long)(hi - lo) * 4 >= p.sort_min) ? snb : nullptr;
-            if (FASTWE && (!EPOK || mode == MODE_WE)) {
+            if constexpr (FAST) {
                 FastLevel f;
                 f.sw = dyn_smem;
-                f.snb = fnb;
-                f.gnb = FAST ? nullptr : nbl;
+                f.gnb = nbl;
                 f.sig = sigma;
                 f.Snext = S + hi;
                 f.cnt = &sm.cnt[L % 3];
@@ -1000,17 +997,12 @@ bc_kernel(KParams p) {
                 forward_we<DIR, NT, LV, !EPOK>(p, lv, sigma, S, bigq, nbl, sb, L, lo, hi, sm, c);
             } else {
                 forward_ep<DIR, NT>(p, lv, sigma, S, L, lo, hi, sm, c);
-                // sigma was accumulated with L2 atomics: drop this SM's L1 lines so the
-                // L1-cached gathers of the next WE level (fast path) see the sums
-                if (FASTWE) __threadfence();
             }
             // (the level functions end with a barrier: every discovery is recorded)
             int nhi;
-            if (FAST && fnb) {
-                // level L+1 = the shared discovery bitmap, written to S in vertex order
-                nhi = hi + compact_level<NT, true>(fnb, p.nb_words, S + hi, sm);
-            } else if (FAST) {
-                nhi = hi + sm.cnt[L % 3];
+            if (FAST && nbl) {
+                // fast path, large level: level L+1 = the bitmap, in vertex order
+                nhi = hi + compact_level<NT>(nbl, p.nb_words, S + hi, sm);
             } else if (LV::BITMAP_DISCOVERY && mode == MODE_WE) {
                 // level L+1 = the discovery bitmap, written to S in vertex order
                 nhi = hi + compact_level<NT>(nb, p.nb_words, S + hi, sm);
@@ -1070,10 +1062,9 @@ bc_kernel(KParams p) {
             const long long t0 = clock64();
             // the forward's successor bits exist only if forward level Lb ran WE
             uint32_t *const sbl = (sb && (!EPOK || modes[Lb] == MODE_WE)) ? sb : nullptr;
-            if (FASTWE && (!EPOK || bmode == MODE_WE)) {
+            if constexpr (FAST) {
                 FastLevel f;
                 f.sw = dyn_smem;
-                f.snb = nullptr;
                 f.gnb = nullptr;
                 f.sig = sigma;
                 f.Snext = nullptr;
@@ -1085,7 +1076,6 @@ bc_kernel(KParams p) {
                 backward_we<NT, LV, !EPOK>(p, lv, sigma, S, bigq, sbl, Lb, blo, bhi, sm, c);
             } else {
                 backward_ep<NT>(p, lv, sigma, omega, S, Lb, blo, bhi, sm, c);
-                if (FASTWE) __threadfence();  // omega written by plain stores; L1 as above
             }
             if (threadIdx.x == 0) {
                 const long long dt = clock64() - t0;

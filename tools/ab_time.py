@@ -24,6 +24,7 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--out", default="gpurun_out/ab")
     ap.add_argument("--compare", nargs=2, default=None)
+    ap.add_argument("--save-max-n", type=int, default=1 << 19, help="save BC vectors only for n <= this")
     a = ap.parse_args()
     if a.compare:
         x, y = np.load(a.compare[0]), np.load(a.compare[1])
@@ -60,11 +61,13 @@ def main():
                 ms.append(bg.stats()["kernel_ms"])
             st = bg.stats()
         name = f"{a.tag}_{key}_{k}_{hashlib.md5(str(sorted(opts.items())).encode()).hexdigest()[:8]}"
-        np.save(os.path.join(a.out, name + ".npy"), out.cpu().numpy())
+        if g.n <= a.save_max_n:
+            np.save(os.path.join(a.out, name + ".npy"), out.cpu().numpy())
         gteps = g.m * src.size / (statistics.median(ms) / 1e3) / 1e9
         print(json.dumps({"tag": a.tag, "config": key, "sources": int(src.size), "opts": opts,
                           "kernel_ms": statistics.median(ms), "all_ms": ms, "gteps": gteps,
-                          "engines": st["engines"], "file": name}), flush=True)
+                          "engines": st["engines"], "phase_cycles": st["phase_cycles"], "levels": st["levels"],
+                          "arcs_scanned": st["arcs_scanned"], "file": name}), flush=True)
 
 
 if __name__ == "__main__":

@@ -21,11 +21,12 @@ def main():
     ap.add_argument("--out", default="profiles/traffic.json")
     a = ap.parse_args()
     out = subprocess.run(["ncu", "-i", a.rep, "--csv", "--page", "raw", "--metrics",
-                          "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum"],
+                          "dram__bytes_read.sum,dram__bytes_write.sum,lts__t_bytes.sum,gpu__time_duration.sum"],
                          capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     h = rows[0]
     dram = 0.0
+    lts = 0.0
     dur = 0.0
     kernels = 0
     for r in rows[2:]:
@@ -36,6 +37,8 @@ def main():
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
         for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
             dram += float(d[k]) * scale.get(rows[1][h.index(k)], 1)
+        if "lts__t_bytes.sum" in d and d["lts__t_bytes.sum"] not in ("", "n/a"):
+            lts += float(d["lts__t_bytes.sum"]) * scale.get(rows[1][h.index("lts__t_bytes.sum")], 1)
         dur += float(d["gpu__time_duration.sum"])
     st = json.load(open(a.stats))
     res = json.load(open(a.out)) if os.path.exists(a.out) else {}
@@ -43,6 +46,8 @@ def main():
                          "bc_kernel_launches_captured": kernels, "dram_bytes": dram,
                          "alg_bytes": st["alg_bytes_per_step"],
                          "dram_bytes_per_alg_byte": dram / st["alg_bytes_per_step"],
+                         "lts_bytes": lts, "lts_bytes_per_alg_byte": (lts / st["alg_bytes_per_step"]) if lts else None,
+                         "kernel_ms_under_ncu": dur / 1e6,
                          "source": os.path.basename(a.rep)}
     json.dump(res, open(a.out, "w"), indent=1)
     print(json.dumps(res[st["config"]]))
