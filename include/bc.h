@@ -155,6 +155,9 @@ typedef struct bc_stats {
     int64_t dist_sum;         /* sum over sources s of sum_t d(s,t) over the reached t: with
                                  n_reached and sources it gives the self-check
                                  sum_v BC(v) = h (dist_sum - n_reached + sources) */
+    int64_t handovers;        /* Alg. 4 / Alg. 5 runs on the fast work-efficient kernel: sources
+                                 whose selector picked an EP level and were therefore re-run
+                                 from scratch by the EP-capable kernel (0 if none)             */
 } bc_stats;
 
 /* Copy a CSR graph to `device` and allocate the per-source workspace.

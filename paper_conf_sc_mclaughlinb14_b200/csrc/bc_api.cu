@@ -112,6 +112,7 @@ struct bc_graph {
     uint32_t *sbits = nullptr;
     int code_words = 0, fb_words = 0;
     int seq_max_deg = 32;
+    int max_deg = 0;      // largest out-degree of the graph
     int warp_max_deg = 4096;
     // graph
     char *graph_buf = nullptr;          // ro | col | src
@@ -136,6 +137,10 @@ struct bc_graph {
     // per-call buffers
     int *src_buf = nullptr;
     long long src_cap = 0;
+    int *fb_src = nullptr;                   // sources handed from the WE-only to the EP kernel
+    long long fb_cap = 0;
+    unsigned long long *fb_n = nullptr;      // [0] handed over, [1] work counter of the EP launch
+    int fb_used = 0;                         // the last compute call used the hand-over path
     double *bc_buf = nullptr;
     unsigned long long *counters = nullptr;  // [0] sampling phase, [1] main phase
     int *keys = nullptr;
@@ -333,7 +338,9 @@ static int configure(bc_graph *g) {
 // most nnz / (warp_max + 1) rows, warp_max being the EFFECTIVE threshold configure() derived
 // (max(seq_max_deg, warp_max_deg)), so the stride must follow every change of either knob.
 static size_t big_stride(const bc_graph *g) {
-    return (((size_t)g->nnz / ((size_t)g->warp_max_deg + 1) + 2) + 31) & ~(size_t)31;
+    // CTA rows (> warp_max) from the front and medium rows (> seq_max, fast path) from the
+    // back: a level holds at most nnz / (seq_max + 1) of them together
+    return (((size_t)g->nnz / ((size_t)g->seq_max_deg + 1) + 2) + 31) & ~(size_t)31;
 }
 
 static int alloc_workspace(bc_graph *g) {
@@ -693,6 +700,8 @@ extern "C" void bc_destroy(bc_graph *g) {
     cudaFree(g->icol);
     cudaFree(g->isrc);
     cudaFree(g->src_buf);
+    cudaFree(g->fb_src);
+    cudaFree(g->fb_n);
     cudaFree(g->bc_buf);
     cudaFree(g->counters);
     cudaFree(g->keys);
@@ -752,6 +761,7 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col_in) 
         for (int v = 0; v <= n; ++v) ro32[v] = (int)ro64[v];
     }
     g->h_ro = ro32;
+    for (int v = 0; v < n; ++v) g->max_deg = std::max(g->max_deg, ro32[v + 1] - ro32[v]);
     CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&g->done, cudaEventDisableTiming));
     for (auto &e : g->tev) CK(cudaEventCreate(&e));
@@ -793,6 +803,7 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col_in) 
         }
     }
     CK(cudaMalloc(&g->counters, 3 * sizeof(unsigned long long)));
+    CK(cudaMalloc(&g->fb_n, 2 * sizeof(unsigned long long)));
     CK(cudaMalloc(&g->keys, sizeof(int) * 8192));
     CK(cudaMalloc(&g->flag, sizeof(int)));
     CK(cudaMemset(g->flag, 0, sizeof(int)));
@@ -929,6 +940,7 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     p.stride_sb = (size_t)g->sb_words;
     p.sb_words = g->sb_words;
     p.seq_max_deg = g->seq_max_deg;
+    p.medq = g->max_deg > g->seq_max_deg ? 1 : 0;
     p.warp_max_deg = g->warp_max_deg;
     p.stats = g->stats;
     p.sampled_flag = g->flag;
@@ -936,36 +948,9 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     return p;
 }
 
-static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
-    if (p0.k <= 0) return BC_OK;
-    if (group_wanted(g, p0)) {
-        const int rc = launch_group(g, p0, st);
-        if (rc == BC_OK || g->opt.engine == BC_ENGINE_GROUP) return rc;
-        free_group(g);
-        g->gr.failed = 1;  // auto: e.g. no memory for the group workspace -> per-source engine
-        cudaGetLastError();
-    }
-    KParams p = p0;
-    // An EP level needs a frontier of >= ep_min_frontier (Alg. 5 guard) or > beta
-    // (Alg. 4) vertices; when no frontier can be that large, the work-efficient-only
-    // kernel (no EP code, no bitmap) is launched instead.
-    const bool ep_possible =
-        !p.skip_if_ep &&
-        (p.launch_mode == LM_EP ||
-         (p.launch_mode == LM_SAMPLED && (long long)p.ep_min_frontier <= (long long)g->n) ||
-         (p.launch_mode == LM_HYBRID && (long long)p.beta < (long long)g->n));
-    // Alg. 5 run whose decision is still on the device: enqueue BOTH kernels, each gated on
-    // the flag (the other exits at once), so a WE decision runs the WE-only kernel and never
-    // pays for the EP code path (the selectors taxed WE levels 2x).
-    if (ep_possible && p.launch_mode == LM_SAMPLED && p.sampled_flag && !p.skip_if_we) {
-        KParams pw = p;
-        pw.skip_if_ep = 1;
-        int rc = launch(g, pw, st);
-        if (rc) return rc;
-        p.skip_if_we = 1;
-    }
-    const bc_graph::KCfg &c = ep_possible ? g->cfg_ep : g->cfg_we;
-    p.fb_words = ep_possible ? g->fb_words : 0;
+// Raw launch of bc_kernel with configuration c (grid = resident CTAs, at most k).
+static int launch_cfg(bc_graph *g, KParams p, const bc_graph::KCfg &c, bool ep_kernel, cudaStream_t st) {
+    p.fb_words = ep_kernel ? g->fb_words : 0;
     const long long cap = std::min<long long>(g->slots, (long long)c.per_sm * g->num_sms);
     const int grid = (int)std::min<long long>(cap, p.k);
     void *args[] = {&p};
@@ -990,6 +975,70 @@ static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
     return BC_OK;
 }
 
+// Whether cfg_we is the fast-path kernel (bc_fast.cuh), which can hand a source whose
+// selector asks for an EP level over to an EP-capable launch.
+static bool we_kernel_is_fast(const bc_graph *g) { return g->lstore == 2 && !g->directed && !g->succ_bits; }
+
+static int launch(bc_graph *g, const KParams &p0, cudaStream_t st) {
+    if (p0.k <= 0) return BC_OK;
+    if (group_wanted(g, p0)) {
+        const int rc = launch_group(g, p0, st);
+        if (rc == BC_OK || g->opt.engine == BC_ENGINE_GROUP) return rc;
+        free_group(g);
+        g->gr.failed = 1;  // auto: e.g. no memory for the group workspace -> per-source engine
+        cudaGetLastError();
+    }
+    KParams p = p0;
+    // An EP level needs a frontier of >= ep_min_frontier (Alg. 5 guard) or > beta
+    // (Alg. 4) vertices; when no frontier can be that large, the work-efficient-only
+    // kernel (no EP code, no bitmap) is launched instead.
+    const bool ep_possible =
+        !p.skip_if_ep &&
+        (p.launch_mode == LM_EP ||
+         (p.launch_mode == LM_SAMPLED && (long long)p.ep_min_frontier <= (long long)g->n) ||
+         (p.launch_mode == LM_HYBRID && (long long)p.beta < (long long)g->n));
+    if (!ep_possible) return launch_cfg(g, p, g->cfg_we, false, st);
+    // Alg. 4 / Alg. 5 run that MAY ask for EP levels: optimistic work-efficient launch.  The
+    // fast WE-only kernel runs every source; a source whose selector picks EP for its next
+    // level is abandoned before its backward stage (nothing of it reaches bc) and queued; an
+    // EP-capable launch then runs the queued sources from scratch with the same selector.  A
+    // run that never picks EP (Alg. 4 on high-diameter graphs, Alg. 5 with a WE decision)
+    // therefore never pays for the EP code path (the selectors taxed WE levels).
+    if ((p.launch_mode == LM_HYBRID || p.launch_mode == LM_SAMPLED) && we_kernel_is_fast(g) && !p.dbg_d &&
+        !p.k_dev && !p.skip_if_we) {
+        if (p.k > g->fb_cap) {
+            cudaFree(g->fb_src);
+            g->fb_src = nullptr;
+            g->fb_cap = 0;
+            CK(cudaMalloc(&g->fb_src, sizeof(int) * (size_t)p.k));
+            g->fb_cap = p.k;
+        }
+        CK(cudaMemsetAsync(g->fb_n, 0, 2 * sizeof(unsigned long long), st));
+        g->fb_used = 1;
+        KParams pw = p;
+        pw.fallback_src = g->fb_src;
+        pw.fallback_n = g->fb_n;
+        int rc = launch_cfg(g, pw, g->cfg_we, false, st);
+        if (rc) return rc;
+        KParams pe = p;
+        pe.sources = g->fb_src;  // caller ids
+        pe.src_base = 0;
+        pe.k_dev = reinterpret_cast<const long long *>(g->fb_n);
+        pe.work_counter = g->fb_n + 1;
+        return launch_cfg(g, pe, g->cfg_ep, true, st);
+    }
+    // Otherwise (other level stores): an Alg. 5 run whose decision is still on the device
+    // enqueues BOTH kernels, each gated on the flag (the other exits at once).
+    if (p.launch_mode == LM_SAMPLED && p.sampled_flag && !p.skip_if_we) {
+        KParams pw = p;
+        pw.skip_if_ep = 1;
+        int rc = launch_cfg(g, pw, g->cfg_we, false, st);
+        if (rc) return rc;
+        p.skip_if_we = 1;
+    }
+    return launch_cfg(g, p, g->cfg_ep, true, st);
+}
+
 // Enqueue one full BC computation on `st`.  d_sources may be NULL (all n).
 static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, double *d_bc,
                            cudaStream_t st) {
@@ -1009,6 +1058,7 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
     g->tev_used[0] = g->tev_used[1] = 0;
     g->batch_ran = 0;
     g->engines = 0;
+    g->fb_used = 0;
     KParams p = base_params(g, acc_bc);
     p.sources = d_sources;
     int rc = BC_OK;
@@ -1379,6 +1429,12 @@ extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {
     st->engines = g->engines;
     st->pad_ = 0;
     st->dist_sum = (int64_t)h.dist_sum;
+    st->handovers = 0;
+    if (g->fb_used) {
+        unsigned long long fb = 0;
+        CK(cudaMemcpy(&fb, g->fb_n, sizeof(fb), cudaMemcpyDeviceToHost));
+        st->handovers = (int64_t)fb;
+    }
     st->kernel_ms = 0.0;
     for (int i = 0; i < 2; ++i)
         if (g->tev_used[i]) {

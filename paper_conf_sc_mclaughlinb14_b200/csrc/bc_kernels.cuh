@@ -69,6 +69,8 @@ struct KParams {
     const long long *k_dev;           // non-NULL: k is read from device memory (batch overflows)
     int skip_if_ep;                   // 1: do nothing when Alg. 5 chose EP (batched / EP-capable kernel runs)
     int skip_if_we;                   // 1: do nothing when Alg. 5 chose WE (the WE-only kernel runs)
+    int *fallback_src;                // fast WE-only kernel: sources whose selector picks an EP
+    unsigned long long *fallback_n;   // level are abandoned and appended here (caller ids)
     unsigned long long *work_counter;
     // workspace (slot-major)
     int *d;                           // GlobalLevels only
@@ -78,7 +80,7 @@ struct KParams {
     int *ends;
     unsigned char *modes;
     int *bigq;           // rows queued for CTA-cooperative expansion (per slot)
-    size_t stride_big;
+    size_t stride_big;   // per-slot bigq entries: CTA rows from the front, medium rows from the back
     size_t stride_n;     // elements per slot for d/sigma/omega/S
     size_t stride_e;     // elements per slot for ends/modes
     double *bc;
@@ -96,6 +98,8 @@ struct KParams {
     size_t stride_sb;
     int sb_words;        // multiple of 4
     int seq_max_deg;     // rows up to this degree: owner thread, CSR order
+    int medq;            // fast path: rows in (seq_max_deg, warp_max_deg] are queued and dealt to
+                         // warps dynamically after the one-thread rows (graph has such rows)
     int warp_max_deg;    // rows up to this degree: one warp; longer: whole CTA
     // strategy
     int launch_mode;
@@ -156,6 +160,7 @@ struct Smem {
     long long idx;
     int cnt[3];           // level L appends at S[hi + cnt[L % 3]] (triple-buffered, see kernel)
     int nbig;             // rows queued for CTA-cooperative expansion in this tile
+    int medc[2], medn[2]; // fast path: medium rows queued / grabbed, by pass parity
     int gw0, gwn;         // row_pass chunk distribution: this CTA's first warp index, warps
                           // sharing the pass (0 / NT/32, except in the group engine's backward)
     int goff;             // group engine: this CTA's offset in the level being compacted
@@ -950,7 +955,9 @@ bc_kernel(KParams p) {
         sm.st = CtaStats{};
         sm.gw0 = 0;
         sm.gwn = NT / 32;
+        sm.medc[0] = sm.medc[1] = sm.medn[0] = sm.medn[1] = 0;
     }
+    int fpass = 0;  // fast-path passes so far (medium-queue counters alternate by parity)
 
     for (;;) {
         if (threadIdx.x == 0) sm.idx = (long long)atomicAdd(p.work_counter, 1ULL);
@@ -958,7 +965,11 @@ bc_kernel(KParams p) {
         const long long idx = sm.idx;
         if (idx >= K) break;
         int s = p.sources ? p.sources[p.src_base + idx] : (int)(p.src_base + idx);
+        const int s_caller = s;
         if (p.perm) s = p.perm[s];  // caller's id -> internal id
+        // per-source statistics (thread 0), rolled back if the source is handed over
+        const unsigned long long sv_lv = sm.st.lv[0], sv_cyc = sm.st.cyc[0], sv_dsum = sm.st.dsum;
+        bool handed_over = false;
         // Alg. 1; all other entries are already unvisited / zero.
         if (threadIdx.x == 0) {
             lv.set_source(s);
@@ -991,7 +1002,7 @@ bc_kernel(KParams p) {
                 f.kmatch = LV::key(L - 1);
                 f.knew = LV::key(L + 1);
                 const unsigned before = c.scanned;
-                fast_pass<NT, true>(p, f, S, lo, hi, L, bigq, sm, c);
+                fast_pass<NT, true>(p, f, S, lo, hi, L, bigq, sm, c, fpass++ & 1);
                 c.arcs_reached += c.scanned - before;
             } else if (!EPOK || mode == MODE_WE) {
                 forward_we<DIR, NT, LV, !EPOK>(p, lv, sigma, S, bigq, nbl, sb, L, lo, hi, sm, c);
@@ -1033,9 +1044,27 @@ bc_kernel(KParams p) {
             }
             if (nhi == hi) break;  // Q_next_len == 0 (Alg. 2 l.11)
             mode = next_mode(p, mode, run_ep, hi - lo, nhi - hi);
+            if (FAST && mode == MODE_EP && p.fallback_src) {
+                // the selector asks for an EP level this WE-only kernel cannot run: hand the
+                // source over to the EP-capable launch (uniform decision over the CTA)
+                handed_over = true;
+                break;
+            }
             lo = hi;
             hi = nhi;
             ++L;
+        }
+        if (handed_over) {
+            if (threadIdx.x == 0) {
+                p.fallback_src[atomicAdd(p.fallback_n, 1ull)] = s_caller;
+                sm.st.lv[0] = sv_lv;
+                sm.st.cyc[0] = sv_cyc;
+                sm.st.dsum = sv_dsum;
+            }
+            c = Counters{};
+            lv.template reset_all<NT>(p.code_words);  // sigma needs no reset (written before read)
+            __syncthreads();
+            continue;
         }
         const int maxdepth = L;
         const int S_len = hi;
@@ -1071,7 +1100,7 @@ bc_kernel(KParams p) {
                 f.cnt = nullptr;
                 f.kmatch = LV::key(Lb + 1);
                 f.knew = 0;
-                fast_pass<NT, false>(p, f, S, blo, bhi, Lb, bigq, sm, c);
+                fast_pass<NT, false>(p, f, S, blo, bhi, Lb, bigq, sm, c, fpass++ & 1);
             } else if (!EPOK || bmode == MODE_WE) {
                 backward_we<NT, LV, !EPOK>(p, lv, sigma, S, bigq, sbl, Lb, blo, bhi, sm, c);
             } else {

@@ -59,7 +59,7 @@ int main(void){
   printf("%zu %zu %zu\n", offsetof(bc_stats, sampling_ep), offsetof(bc_stats, inflight),
          offsetof(bc_stats, kernel_ms));
   printf("%zu %zu %d\n", offsetof(bc_options, engine), offsetof(bc_options, group_ctas), BC_ENGINE_GROUP);
-  printf("%zu\n", offsetof(bc_stats, dist_sum));
+  printf("%zu %zu\n", offsetof(bc_stats, dist_sum), offsetof(bc_stats, handovers));
   return 0; }
 """
     import tempfile
@@ -72,7 +72,7 @@ int main(void){
     O, S = _bc.bc_options, _bc.bc_stats
     assert vals == [ctypes.sizeof(O), O.gamma.offset, O.level_store.offset, ctypes.sizeof(S),
                     S.sampling_ep.offset, S.inflight.offset, S.kernel_ms.offset,
-                    O.engine.offset, O.group_ctas.offset, _bc.ENGINES["group"], S.dist_sum.offset]
+                    O.engine.offset, O.group_ctas.offset, _bc.ENGINES["group"], S.dist_sum.offset, S.handovers.offset]
 
 
 def test_default_options_are_the_papers(lib):

@@ -475,3 +475,31 @@ def test_seq_max_deg_shrink_reallocates_bigq(bcmod, oracle_mod):
         check_bc(bg, g, src, oracle_mod)
         bg.set_options(seq_max_deg=4, warp_max_deg=8)
         check_bc(bg, g, src, oracle_mod)
+
+
+@pytest.mark.parametrize("key,strategy,expect_handover", [
+    ("c3", "hybrid", False),     # Alg. 4 never picks EP on RGG (frontier changes < alpha)
+    ("c2", "sampling", False),   # Alg. 5 decides WE on the lattice (median depth >= 64)
+    ("c4", "hybrid", True),      # Alg. 4 picks EP for the Kronecker middle levels
+    ("c4", "sampling", True),    # Alg. 5 decides EP; guard 512 admits EP levels
+])
+def test_optimistic_we_with_handover(bcmod, oracle_mod, key, strategy, expect_handover):
+    """Alg. 4 / Alg. 5 with the paper's parameters run on the fast work-efficient kernel;
+    a source whose selector picks an EP level is handed over (re-run from scratch) to the
+    EP-capable kernel.  BC is the oracle's either way, every source is counted once, and the
+    per-level modes of a handed-over source match the selector replay."""
+    from oracle import selectors as sel
+    g = graph(key)
+    src = gg.CONFIGS[key].sources(g)[:900] if gg.CONFIGS[key].k else gg.sample_sources(g, 900, seed=12)
+    with bcmod.BCGraph.from_graph(g, strategy=strategy) as bg:
+        check_bc(bg, g, src, oracle_mod, nthreads=16)
+        st = bg.stats()
+        assert st["sources"] == src.size
+        if expect_handover:
+            assert st["handovers"] > 0 and st["ep_levels"] > 0
+        else:
+            assert st["handovers"] == 0 and st["ep_levels"] == 0
+        if strategy == "hybrid":
+            for s in src[:3]:
+                ref = oracle_mod.single_source(g, int(s))
+                assert bg.single_source(int(s))["level_modes"].tolist() == sel.hybrid_modes(ref["level_sizes"].tolist())
