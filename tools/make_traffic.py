@@ -39,7 +39,8 @@ def main():
             dram += float(d[k]) * scale.get(rows[1][h.index(k)], 1)
         if "lts__t_bytes.sum" in d and d["lts__t_bytes.sum"] not in ("", "n/a"):
             lts += float(d["lts__t_bytes.sum"]) * scale.get(rows[1][h.index("lts__t_bytes.sum")], 1)
-        dur += float(d["gpu__time_duration.sum"])
+        tunit = rows[1][h.index("gpu__time_duration.sum")]
+        dur += float(d["gpu__time_duration.sum"]) * {"nsecond": 1e-6, "ns": 1e-6, "usecond": 1e-3, "us": 1e-3, "msecond": 1.0, "ms": 1.0, "second": 1e3, "s": 1e3}.get(tunit, 1.0)
     st = json.load(open(a.stats))
     res = json.load(open(a.out)) if os.path.exists(a.out) else {}
     res[st["config"]] = {"strategy": st["strategy"], "sources": st["sources"],
@@ -47,7 +48,7 @@ def main():
                          "alg_bytes": st["alg_bytes_per_step"],
                          "dram_bytes_per_alg_byte": dram / st["alg_bytes_per_step"],
                          "lts_bytes": lts, "lts_bytes_per_alg_byte": (lts / st["alg_bytes_per_step"]) if lts else None,
-                         "kernel_ms_under_ncu": dur / 1e6,
+                         "kernel_ms_under_ncu": dur,
                          "source": os.path.basename(a.rep)}
     json.dump(res, open(a.out, "w"), indent=1)
     print(json.dumps(res[st["config"]]))
