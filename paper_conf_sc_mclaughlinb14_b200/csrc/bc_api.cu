@@ -479,15 +479,22 @@ static int group_count(const bc_graph *g, int grid) {
     // small world c5ws is fastest with 4 groups of 74 CTAs (1509 ms; 148 CTAs 1590, 37:
     // 1609), the skewed Kronecker c5k with groups of 12 CTAs (2103 ms; 9: 2149, 6: 2308,
     // 18: 2552).  Skewed = internally relabelled by degree (want_reorder).
-    const int ctas = g->perm ? 12 : std::max(1, grid / 4);
+    const int ctas = g->perm ? 18 : std::max(1, grid / 4);
     return std::max(1, std::min(grid, grid / ctas));
+}
+
+// The group engine's work-efficient levels run through the fast path on degree-relabelled
+// (skewed) graphs and through the generic row_pass otherwise (measured).
+static bool group_fast(const bc_graph *g) {
+    if (const char *e = getenv("BC_GROUP_FAST")) return atoi(e) != 0;  // tuning override
+    return g->perm != nullptr;
 }
 
 static int alloc_group(bc_graph *g) {
     bc_graph::Group &q = g->gr;
     const int nt = g->n >= (1 << 17) ? 512 : 256;
     int per_sm = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bcgroup::group_kernel_fn(nt), nt, 0));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bcgroup::group_kernel_fn(nt, group_fast(g)), nt, 0));
     if (per_sm < 1) return fail(BC_EINTERNAL, "group kernel cannot be resident");
     const int grid = per_sm * g->num_sms;
     const int G = group_count(g, grid);
@@ -589,7 +596,7 @@ static int launch_group(bc_graph *g, const KParams &p0, cudaStream_t st) {
     }
     lc.attrs = attr;
     lc.numAttrs = na;
-    CK(cudaLaunchKernelExC(&lc, bcgroup::group_kernel_fn(q.nt), args));
+    CK(cudaLaunchKernelExC(&lc, bcgroup::group_kernel_fn(q.nt, group_fast(g)), args));
     CK(cudaGetLastError());
     g->launches++;
     g->bc_launches++;

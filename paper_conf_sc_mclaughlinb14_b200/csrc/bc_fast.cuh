@@ -1,6 +1,8 @@
-// bc_fast.cuh -- the work-efficient fast path of bc_kernel for undirected graphs whose 2-bit
-// level codes live in shared memory (bc_kernel<false, SmemCodes, NT, false, false>: every
-// Alg. 5 run with the B200 guard and every WE run on n <= ~2^18, i.e. c1..c4).
+// bc_fast.cuh -- the work-efficient fast path for undirected graphs with 2-bit level codes:
+//  * G = false: codes in shared memory, bc_kernel<false, SmemCodes, NT, false, false> (every
+//    work-efficient launch on n <= ~2^18, i.e. c1..c4);
+//  * G = true: codes in global memory (L1-cached reads), the group engine (bc_group.cu, c5),
+//    with idempotent discovery marks and the successor bitmap over arcs.
 //
 // Same arithmetic, same order and same outputs as the generic row_pass / forward_we /
 // backward_we (Alg. 2 l.3-8 as a pull; Alg. 3 l.5-9; Eq. 3),
@@ -50,15 +52,25 @@ __device__ __forceinline__ uint32_t atom_or_shared_if(uint32_t *addr, uint32_t v
 
 // Per-level context of the fast path.
 struct FastLevel {
-    uint32_t *sw;      // shared 2-bit codes
+    uint32_t *sw;      // 2-bit codes (shared memory if !G, global memory if G)
     uint32_t *gnb;     // non-null: discoveries go to this level bitmap ONLY (no S append); the
                        // kernel rebuilds level L+1 from it in vertex order (sorted frontiers)
+    uint32_t *sb;      // G: successor bits over CSR positions (nullptr = off; Jia et al.'s O(m)
+                       // boolean array): the forward marks the DAG successor arcs, the
+                       // backward visits only them (no code probe, columns only for them)
     double *sig;       // sigma (forward) / sigma-then-omega (backward), this slot
     int *Snext;        // S + hi: where level L+1 is appended (queue mode)
     int *cnt;          // &sm.cnt[L % 3]
     int kmatch;        // forward: key(L-1) (predecessors); backward: key(L+1) (successors)
     int knew;          // forward: key(L+1), the code a discovery sets (as a 2-bit value)
 };
+
+template <bool G>
+__device__ __forceinline__ int fcode(const FastLevel &f, int u) {
+    if (!G) return code_at(f.sw, u);
+    const uint32_t wd = __ldca(&f.sw[(unsigned)u >> 4]);  // L1: invalidated at every level start
+    return (int)(__funnelshift_r(wd, wd, (unsigned)u << 1) & 3u);
+}
 
 __device__ __forceinline__ void red_or_global_if(uint32_t *addr, uint32_t val, bool c) {
     asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.global.or.b32 [%0], %1;\n\t}"
@@ -67,11 +79,22 @@ __device__ __forceinline__ void red_or_global_if(uint32_t *addr, uint32_t val, b
                  : "memory");
 }
 
-// Claims of up to four neighbours (forward only): predicated shared atomics on the code
-// words; winners are marked in the level bitmap (large levels: the kernel rebuilds level
-// L+1 from it in vertex order) or appended to S with ONE warp scan and ONE shared atomic
-// for all four slots.  Warp-uniform call.
+// Claims of up to four neighbours (forward only), warp-uniform call.
+//  !G: predicated shared atomics on the code words; winners are marked in the level bitmap
+//      (large levels: the kernel rebuilds level L+1 from it in vertex order) or appended to
+//      S with ONE warp scan and ONE shared atomic for all four slots.
+//   G: no winner election: every claimer ORs the code and the level bitmap (idempotent,
+//      fire-and-forget); the group engine compacts level L+1 from the bitmap.
+template <bool G>
 __device__ __forceinline__ void fast_claims(const FastLevel &f, const int (&u)[4], const bool (&un)[4]) {
+    if (G) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            red_or_global_if(&f.sw[(unsigned)u[j] >> 4], (uint32_t)f.knew << (((unsigned)u[j] << 1) & 30u), un[j]);
+            red_or_global_if(&f.gnb[(unsigned)u[j] >> 5], 1u << (u[j] & 31), un[j]);
+        }
+        return;
+    }
     bool won[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
@@ -102,19 +125,65 @@ __device__ __forceinline__ void fast_claims(const FastLevel &f, const int (&u)[4
         if (won[j]) f.Snext[base++] = u[j];
 }
 
+// Successor-bit window of a one-thread row: bits of words w0, w0 + 1 (64 arcs).
+__device__ __forceinline__ void sb_flush(uint32_t *sb, int w0, uint64_t win) {
+    red_or_global_if(&sb[w0], (uint32_t)win, (uint32_t)win != 0u);
+    red_or_global_if(&sb[w0 + 1], (uint32_t)(win >> 32), (win >> 32) != 0ull);
+}
+__device__ __forceinline__ uint64_t sb_window(const uint32_t *sb, int w0, int end, bool any) {
+    uint64_t win = 0;
+    if (any) {
+        win = __ldcg(&sb[w0]);
+        if (end > (w0 + 1) * 32) win |= (uint64_t)__ldcg(&sb[w0 + 1]) << 32;
+    }
+    return win;
+}
+
 // Quads of the one-thread rows of a 32-vertex chunk; lane = row [beg, end) (deg <= seq_max,
 // deg = 0 for lanes without a row).  Warp-uniform trip count.  Returns the lane's sum of
 // gathers in CSR order.
-template <bool FWD>
+template <bool G, bool FWD>
 __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *__restrict__ cols, int beg,
                                                 int end, Counters &c) {
     const int q0 = beg & ~3;
     const int nq = end > beg ? ((end + 3) >> 2) - (beg >> 2) : 0;
     const int maxq = __reduce_max_sync(FULL, (unsigned)nq);
     double acc = 0.0;
+    const bool bits = G && f.sb;
+    if (bits && !FWD) {
+        // backward: only the successor arcs the forward marked; no probe
+        // (per-lane trip count: no warp collective in here, and a lane whose quads hold no
+        // successor skips them)
+        int w0 = beg >> 5;
+        uint64_t win = sb_window(f.sb, w0, end, nq > 0);
+        for (int q = 0; q < nq; ++q) {
+            const int pos = q0 + 4 * q;
+            int off = pos - 32 * w0;
+            if (off >= 64) {
+                w0 += 2;
+                off -= 64;
+                win = sb_window(f.sb, w0, end, true);
+            }
+            unsigned valid = 0xFu;
+            if (pos < beg) valid &= 0xFu << (beg - pos);
+            if (pos + 4 > end) valid &= 0xFu >> min(4, pos + 4 - end);
+            const unsigned sbits = (unsigned)(win >> off) & valid;
+            if (!sbits) continue;
+            const int4 c4 = *reinterpret_cast<const int4 *>(cols + pos);
+            const int u[4] = {c4.x, c4.y, c4.z, c4.w};
+            double g[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) g[j] = ldca_if(f.sig + u[j], (sbits >> j) & 1u);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) acc += g[j];
+        }
+        return acc;
+    }
     int4 nx = make_int4(0, 0, 0, 0);
     if (nq > 0) nx = *reinterpret_cast<const int4 *>(cols + q0);
     unsigned dag = 0;
+    int w0 = beg >> 5;
+    uint64_t win = 0;
     for (int q = 0; q < maxq; ++q) {
         const int pos = q0 + 4 * q;
         const int4 c4 = nx;
@@ -127,7 +196,7 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
         const int u[4] = {c4.x, c4.y, c4.z, c4.w};
         int k[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) k[j] = code_at(f.sw, u[j]);
+        for (int j = 0; j < 4; ++j) k[j] = fcode<G>(f, u[j]);
         bool pg[4];
         double g[4];
 #pragma unroll
@@ -143,12 +212,26 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
                 un[j] = ((valid >> j) & 1u) && k[j] == 0;
                 any |= un[j];
             }
-            if (__any_sync(FULL, any)) fast_claims(f, u, un);
+            if (__any_sync(FULL, any)) fast_claims<G>(f, u, un);
             dag += (unsigned)pg[0] + (unsigned)pg[1] + (unsigned)pg[2] + (unsigned)pg[3];
+            if (bits) {  // successors: unvisited or already on level L+1
+                int off = pos - 32 * w0;
+                if (off >= 64) {
+                    sb_flush(f.sb, w0, win);
+                    w0 += 2;
+                    off -= 64;
+                    win = 0;
+                }
+                unsigned sm4 = 0;
+#pragma unroll
+                for (int j = 0; j < 4; ++j) sm4 |= (((valid >> j) & 1u) && (k[j] == 0 || k[j] == f.knew)) ? 1u << j : 0u;
+                win |= (uint64_t)sm4 << off;
+            }
         }
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc += g[j];
     }
+    if (FWD && bits) sb_flush(f.sb, w0, win);
     if (FWD) c.dag += dag;
     return acc;
 }
@@ -156,14 +239,50 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
 // One row [b, e) expanded by `stride` cooperating threads (a warp or the CTA), thread t
 // taking arcs t, t + stride, ... (four in flight).  Warp-uniform within each warp.  Returns
 // the thread's partial sum (the caller reduces).
-//
-// (Successor bits for these rows -- forward ballots + REDs marking the DAG arcs, backward
-// visiting only marked arcs -- were measured slower on B200: c4 161 -> 188 ms per 4,096
-// sources, the forward paying more than the backward saved.)
-template <bool FWD>
+// (With codes in shared memory, successor bits for these rows were measured slower on B200:
+// c4 161 -> 188 ms per 4,096 sources, the forward paying more than the backward saved; the
+// group engine, whose probes are global loads, keeps them.)
+template <bool G, bool FWD>
 __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *__restrict__ cols, int b, int e,
                                                 int t, int stride, Counters &c) {
     double acc = 0.0;
+    const int lane = threadIdx.x & 31;
+    const bool bits = G && f.sb;
+    if (bits && !FWD) {
+        uint32_t wn[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int a = b + t + j * stride;
+            wn[j] = a < e ? __ldcg(&f.sb[a >> 5]) : 0u;
+        }
+        for (int base = b; base < e; base += 4 * stride) {
+            bool s[4];
+            int a[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                a[j] = base + t + j * stride;
+                s[j] = a[j] < e && ((wn[j] >> (a[j] & 31)) & 1u);
+            }
+            const int bn = base + 4 * stride;
+            if (bn < e) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const int an = bn + t + j * stride;
+                    wn[j] = an < e ? __ldcg(&f.sb[an >> 5]) : 0u;
+                }
+            }
+            if (!__any_sync(FULL, s[0] | s[1] | s[2] | s[3])) continue;
+            int u[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) u[j] = s[j] ? cols[a[j]] : 0;
+            double g[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) g[j] = ldca_if(f.sig + u[j], s[j]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) acc += g[j];
+        }
+        return acc;
+    }
     unsigned dag = 0;
     int un_[4];
 #pragma unroll
@@ -183,7 +302,7 @@ __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *_
         }
         int k[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) k[j] = code_at(f.sw, u[j]);
+        for (int j = 0; j < 4; ++j) k[j] = fcode<G>(f, u[j]);
         bool pg[4];
         double g[4];
 #pragma unroll
@@ -199,8 +318,20 @@ __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *_
                 un[j] = ok[j] && k[j] == 0;
                 any |= un[j];
             }
-            if (__any_sync(FULL, any)) fast_claims(f, u, un);
+            if (__any_sync(FULL, any)) fast_claims<G>(f, u, un);
             dag += (unsigned)pg[0] + (unsigned)pg[1] + (unsigned)pg[2] + (unsigned)pg[3];
+            if (bits) {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const unsigned m = __ballot_sync(FULL, ok[j] && (k[j] == 0 || k[j] == f.knew));
+                    if (lane == 0 && m) {  // the warp's 32 arcs are consecutive
+                        const int A = base + j * stride + (t - lane);
+                        const int sh = A & 31;
+                        atomicOr(&f.sb[A >> 5], m << sh);  // RED: result unused
+                        if (sh) atomicOr(&f.sb[(A >> 5) + 1], m >> (32 - sh));
+                    }
+                }
+            }
         }
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc += g[j];
@@ -209,17 +340,13 @@ __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *_
     return acc;
 }
 
-// One forward (FWD) or backward level over S[lo, hi): phase A (warps take 32-vertex chunks:
-// one-thread rows, then warp rows one at a time), phase B (rows > warp_max, whole CTA).
-// Forward finish: sigma[v] = sum (L > 0).  Backward finish: finish_dependency (omega in
-// place, bc += delta).  Ends with a CTA barrier (in phase B's test).
-template <bool FWD>
+template <bool G, bool FWD>
 __device__ __forceinline__ void fast_medium_row(const KParams &p, const FastLevel &f, int w, int b, int e, int L,
                                                 Counters &c) {
     const int lane = threadIdx.x & 31;
     double swm = 0.0;
     if (!FWD && lane == 0) swm = __ldcg(&f.sig[w]);
-    const double a = warp_sum(fast_coop_row<FWD>(f, p.col, b, e, lane, 32, c));
+    const double a = warp_sum(fast_coop_row<G, FWD>(f, p.col, b, e, lane, 32, c));
     if (lane == 0) {
         if (FWD) {
             if (L > 0) {
@@ -232,7 +359,13 @@ __device__ __forceinline__ void fast_medium_row(const KParams &p, const FastLeve
     }
 }
 
-template <int NT, bool FWD>
+// One forward (FWD) or backward level over S[lo, hi): phase A (warps take 32-vertex chunks --
+// warp sm.gw0 + wid of sm.gwn sharing the pass -- and sum their one-thread rows, queueing the
+// medium rows), phase M (medium rows dealt to warps dynamically; B200: c4 159.9 -> 154.5 ms
+// per 4,096 sources; graphs without medium rows skip it), phase B (rows > warp_max, whole
+// CTA).  Forward finish: sigma[v] = sum (L > 0).  Backward finish: finish_dependency (omega
+// in place, bc += delta).  Ends with a CTA barrier (in phase B's test).
+template <int NT, bool G, bool FWD>
 __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, const int *__restrict__ S, int lo,
                                           int hi, int L, int *bigq, Smem<NT> &sm, Counters &c, int par) {
     constexpr int NW = NT / 32;
@@ -240,7 +373,8 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
     const int *__restrict__ rows = p.ro;
     const int *__restrict__ cols = p.col;
     const int seq_max = p.seq_max_deg, warp_max = p.warp_max_deg;
-    for (int base = lo + wid * 32; base < hi; base += NT) {
+    const int gstep = sm.gwn * 32;
+    for (int base = lo + (sm.gw0 + wid) * 32; base < hi; base += gstep) {
         const int i = base + lane;
         int v = -1, beg = 0, deg = 0;
         if (i < hi) {
@@ -252,7 +386,7 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
         const bool seq = v >= 0 && deg <= seq_max;
         double sw = 0.0;
         if (!FWD && seq) sw = __ldcg(&f.sig[v]);  // sigma[w], issued early
-        const double acc = fast_seq_rows<FWD>(f, cols, beg, seq ? beg + deg : beg, c);
+        const double acc = fast_seq_rows<G, FWD>(f, cols, beg, seq ? beg + deg : beg, c);
         if (seq) {
             if (FWD) {
                 if (L > 0) f.sig[v] = acc;
@@ -261,9 +395,7 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
             }
         }
         unsigned med = __ballot_sync(FULL, v >= 0 && deg > seq_max && deg <= warp_max);
-        // medium rows go to the CTA's medium queue (back of bigq), dealt out dynamically below
-        // (B200: c4 159.9 -> 154.5 ms per 4,096 sources; graphs without medium rows skip it)
-        if (p.medq && med) {
+        if (p.medq && med) {  // to the CTA's medium queue (back of bigq)
             int q = 0;
             if (lane == 0) q = atomicAdd(&sm.medc[par], __popc(med));
             q = __shfl_sync(FULL, q, 0);
@@ -278,7 +410,7 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
             const int e = b + __shfl_sync(FULL, deg, leader);
             double swm = 0.0;
             if (!FWD && lane == leader) swm = __ldcg(&f.sig[w]);
-            const double a = warp_sum(fast_coop_row<FWD>(f, cols, b, e, lane, 32, c));
+            const double a = warp_sum(fast_coop_row<G, FWD>(f, cols, b, e, lane, 32, c));
             if (lane == leader) {
                 if (FWD) {
                     if (L > 0) {
@@ -302,7 +434,7 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
             r = __shfl_sync(FULL, r, 0);
             if (r >= nmed) break;
             const int w = __ldcg(&bigq[p.stride_big - 1 - r]);
-            fast_medium_row<FWD>(p, f, w, rows[w], rows[w + 1], L, c);
+            fast_medium_row<G, FWD>(p, f, w, rows[w], rows[w + 1], L, c);
         }
     }
     if (__syncthreads_or(sm.nbig > 0)) {
@@ -312,7 +444,7 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
             const int b = rows[v], e = rows[v + 1];
             double swb = 0.0;
             if (!FWD && threadIdx.x == 0) swb = __ldcg(&f.sig[v]);
-            const double a = warp_sum(fast_coop_row<FWD>(f, cols, b, e, threadIdx.x, NT, c));
+            const double a = warp_sum(fast_coop_row<G, FWD>(f, cols, b, e, threadIdx.x, NT, c));
             if (lane == 0) sm.red[wid] = a;
             __syncthreads();
             if (threadIdx.x == 0) {

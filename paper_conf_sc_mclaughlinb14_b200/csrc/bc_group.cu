@@ -124,7 +124,11 @@ __device__ __forceinline__ int group_compact(uint32_t *nb, int words, int r, int
     return total;
 }
 
-template <int NT>
+// FASTG: work-efficient levels through the fast path (bc_fast.cuh, G = true) instead of the
+// generic row_pass.  Measured per graph kind on B200: faster on the skewed,
+// degree-relabelled Kronecker graph (c5k 2100 -> 2024 ms per 2,048 sources; 1954 with 18
+// CTAs per group), slower on the unskewed small world (c5ws 1500 -> 1568 ms, the backward).
+template <int NT, bool FASTG>
 __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p, GParams gp) {
     constexpr int NW = NT / 32;
     __shared__ Smem<NT> sm;
@@ -157,7 +161,22 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
         sm.gw0 = 0;
         sm.gwn = NW;
         sm.cnt[0] = sm.cnt[1] = sm.cnt[2] = 0;
+        sm.medc[0] = sm.medc[1] = sm.medn[0] = sm.medn[1] = 0;
     }
+    int fpass = 0;  // fast-path passes (medium-queue counters alternate by parity)
+    // fast path (bc_fast.cuh, G = true): global codes, idempotent marks, successor bits
+    auto mk = [&](uint32_t *gnb, int kmatch, int knew) {
+        FastLevel f;
+        f.sw = lv.w;
+        f.gnb = gnb;
+        f.sb = sb;
+        f.sig = sigma;
+        f.Snext = nullptr;
+        f.cnt = nullptr;
+        f.kmatch = kmatch;
+        f.knew = knew;
+        return f;
+    };
     const long long K = p.k;
     if (r == 0 && tid == 0) *next_idx = (long long)atomicAdd(p.work_counter, 1ULL);
     group_sync(bar, target, C);
@@ -187,8 +206,17 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
         for (;;) {
             uint32_t *nbw_next = nbb + (size_t)((L + 1) % 3) * nbw;
             // (a) Alg. 2 over this CTA's share of level L (ends with a CTA barrier)
-            if (mycnt > 0)
-                forward_we<false, NT, GlobalCodes, true>(p, lv, sigma, S, bigq, nbw_next, sb, L, mylo, mylo + mycnt, sm, c);
+            if (mycnt > 0) {
+                if constexpr (!FASTG) {
+                    forward_we<false, NT, GlobalCodes, true>(p, lv, sigma, S, bigq, nbw_next, sb, L, mylo,
+                                                             mylo + mycnt, sm, c);
+                } else {
+                    const unsigned before = c.scanned;
+                    fast_pass<NT, true, true>(p, mk(nbw_next, GlobalCodes::key(L - 1), GlobalCodes::key(L + 1)), S,
+                                              mylo, mylo + mycnt, L, bigq, sm, c, fpass++ & 1);
+                    c.arcs_reached += c.scanned - before;
+                }
+            }
             // (b) level L+1 is complete once every CTA got here
             group_sync(bar, target, C);
             const int tot = *(volatile int *)&lvl[L & 3];
@@ -249,14 +277,24 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             const long long t0 = clock64();
             if (Lb < RCAP) {
                 const int2 rg = s_reg[Lb];
-                backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, rg.x, rg.x + rg.y, sm, c);
+                if constexpr (!FASTG) {
+                    backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, rg.x, rg.x + rg.y, sm, c);
+                } else {
+                    fast_pass<NT, true, false>(p, mk(nullptr, GlobalCodes::key(Lb + 1), 0), S, rg.x, rg.x + rg.y, Lb,
+                                               bigq, sm, c, fpass++ & 1);
+                }
             } else {
                 if (tid == 0) {
                     sm.gw0 = r * NW;
                     sm.gwn = C * NW;
                 }
                 __syncthreads();
-                backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, ends[Lb], ends[Lb + 1], sm, c);
+                if constexpr (!FASTG) {
+                    backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, ends[Lb], ends[Lb + 1], sm, c);
+                } else {
+                    fast_pass<NT, true, false>(p, mk(nullptr, GlobalCodes::key(Lb + 1), 0), S, ends[Lb], ends[Lb + 1],
+                                               Lb, bigq, sm, c, fpass++ & 1);
+                }
                 __syncthreads();
                 if (tid == 0) {
                     sm.gw0 = 0;
@@ -314,8 +352,9 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
     }
 }
 
-const void *group_kernel_fn(int nt) {
-    return nt == 256 ? (const void *)group_kernel<256> : (const void *)group_kernel<512>;
+const void *group_kernel_fn(int nt, bool fast) {
+    if (fast) return nt == 256 ? (const void *)group_kernel<256, true> : (const void *)group_kernel<512, true>;
+    return nt == 256 ? (const void *)group_kernel<256, false> : (const void *)group_kernel<512, false>;
 }
 
 }  // namespace bcgroup

@@ -45,6 +45,6 @@ struct GParams {
 // arguments (KParams, GParams).  KParams: sigma / S / ends / gcodes / nbits (3 buffers of
 // nb_words) / sbits are per GROUP (strides stride_n, stride_e, stride_codes, stride_nb,
 // stride_sb); bigq is per CTA (stride_big).
-const void *group_kernel_fn(int nt);
+const void *group_kernel_fn(int nt, bool fast);
 
 }  // namespace bcgroup

@@ -996,13 +996,14 @@ bc_kernel(KParams p) {
                 FastLevel f;
                 f.sw = dyn_smem;
                 f.gnb = nbl;
+                f.sb = nullptr;
                 f.sig = sigma;
                 f.Snext = S + hi;
                 f.cnt = &sm.cnt[L % 3];
                 f.kmatch = LV::key(L - 1);
                 f.knew = LV::key(L + 1);
                 const unsigned before = c.scanned;
-                fast_pass<NT, true>(p, f, S, lo, hi, L, bigq, sm, c, fpass++ & 1);
+                fast_pass<NT, false, true>(p, f, S, lo, hi, L, bigq, sm, c, fpass++ & 1);
                 c.arcs_reached += c.scanned - before;
             } else if (!EPOK || mode == MODE_WE) {
                 forward_we<DIR, NT, LV, !EPOK>(p, lv, sigma, S, bigq, nbl, sb, L, lo, hi, sm, c);
@@ -1095,12 +1096,13 @@ bc_kernel(KParams p) {
                 FastLevel f;
                 f.sw = dyn_smem;
                 f.gnb = nullptr;
+                f.sb = nullptr;
                 f.sig = sigma;
                 f.Snext = nullptr;
                 f.cnt = nullptr;
                 f.kmatch = LV::key(Lb + 1);
                 f.knew = 0;
-                fast_pass<NT, false>(p, f, S, blo, bhi, Lb, bigq, sm, c, fpass++ & 1);
+                fast_pass<NT, false, false>(p, f, S, blo, bhi, Lb, bigq, sm, c, fpass++ & 1);
             } else if (!EPOK || bmode == MODE_WE) {
                 backward_we<NT, LV, !EPOK>(p, lv, sigma, S, bigq, sbl, Lb, blo, bhi, sm, c);
             } else {

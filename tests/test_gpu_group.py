@@ -172,3 +172,20 @@ def test_group_matches_per_source_on_many_sources(bcmod, key):
             out[eng] = (bc, [st[k] for k in ("levels", "n_reached", "arcs_reached", "dag_arcs")])
     assert out["group"][1] == out["per_source"][1]
     assert rel_err(out["group"][0], out["per_source"][0]) <= BC_TOL
+
+
+@pytest.mark.parametrize("fast", ["0", "1"])
+@pytest.mark.parametrize("key,k", [("c1", None), ("c2", 64), ("c4", 96), ("c5ws", 24), ("c5k", 24)])
+def test_generic_and_fast_group_paths(bcmod, oracle_mod, monkeypatch, fast, key, k):
+    """The group engine's two implementations of the work-efficient levels -- the generic
+    row_pass and the fast path (bc_fast.cuh, G = true; auto on degree-relabelled graphs) --
+    on the same graphs, forced with BC_GROUP_FAST: identical d / sigma, BC within 1e-9."""
+    monkeypatch.setenv("BC_GROUP_FAST", fast)
+    g = graph(key)
+    src = None if k is None else (gg.CONFIGS[key].sources(g)[:k] if gg.CONFIGS[key].k
+                                   else gg.sample_sources(g, k, seed=6))
+    with group_graph(bcmod, g, 0, strategy="we") as bg:
+        check_bc(bg, g, src, oracle_mod, nthreads=16)
+        s0 = 5 if src is None else int(src[0])
+        check_source(bg, g, s0, oracle_mod)
+        assert bg.stats()["engines"] & 4
