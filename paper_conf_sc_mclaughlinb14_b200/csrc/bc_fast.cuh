@@ -63,7 +63,27 @@ struct FastLevel {
     int *cnt;          // &sm.cnt[L % 3]
     int kmatch;        // forward: key(L-1) (predecessors); backward: key(L+1) (successors)
     int knew;          // forward: key(L+1), the code a discovery sets (as a 2-bit value)
+#ifdef BC_SMEM_QUEUE
+    int *wqn;          // variant: per-warp staging buffers in shared memory ([NT/32], [NT/32][160])
+    int *wq;
+#endif
 };
+
+#ifdef BC_SMEM_QUEUE
+// variant: flush this warp's staged discoveries to S (one shared atomic, coalesced stores)
+__device__ __forceinline__ void wq_flush(const FastLevel &f) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int n0 = f.wqn[wid];
+    if (n0 == 0) return;
+    int base = 0;
+    if (lane == 0) base = atomicAdd(f.cnt, n0);
+    base = __shfl_sync(FULL, base, 0);
+    for (int i = lane; i < n0; i += 32) f.Snext[base + i] = f.wq[wid * 160 + i];
+    __syncwarp();
+    if (lane == 0) f.wqn[wid] = 0;
+    __syncwarp();
+}
+#endif
 
 template <bool G>
 __device__ __forceinline__ int fcode(const FastLevel &f, int u) {
@@ -117,6 +137,20 @@ __device__ __forceinline__ void fast_claims(const FastLevel &f, const int (&u)[4
     }
     const int tot = __shfl_sync(FULL, incl, 31);
     if (tot == 0) return;
+#ifdef BC_SMEM_QUEUE
+    {
+        const int wid = threadIdx.x >> 5;
+        if (f.wqn[wid] + tot > 160) wq_flush(f);
+        int pos = f.wqn[wid] + incl - cnt;
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+            if (won[j]) f.wq[wid * 160 + pos++] = u[j];
+        __syncwarp();
+        if (lane == 31) f.wqn[wid] += tot;
+        __syncwarp();
+        return;
+    }
+#endif
     int base = 0;
     if (lane == 31) base = atomicAdd(f.cnt, tot);
     base = __shfl_sync(FULL, base, 31) + incl - cnt;
@@ -464,6 +498,12 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
             __syncthreads();
         }
     }
+#ifdef BC_SMEM_QUEUE
+    if (FWD && !G && !f.gnb) {
+        wq_flush(f);
+        __syncthreads();
+    }
+#endif
 }
 
 }  // namespace bcdev
