@@ -161,10 +161,6 @@ struct Smem {
     int cnt[3];           // level L appends at S[hi + cnt[L % 3]] (triple-buffered, see kernel)
     int nbig;             // rows queued for CTA-cooperative expansion in this tile
     int medc[2], medn[2]; // fast path: medium rows queued / grabbed, by pass parity
-#ifdef BC_SMEM_QUEUE
-    int wqn[NT / 32];     // variant: per-warp staging of discoveries in shared memory
-    int wq[NT / 32][160];
-#endif
     int gw0, gwn;         // row_pass chunk distribution: this CTA's first warp index, warps
                           // sharing the pass (0 / NT/32, except in the group engine's backward)
     int goff;             // group engine: this CTA's offset in the level being compacted
@@ -961,9 +957,6 @@ bc_kernel(KParams p) {
         sm.gwn = NT / 32;
         sm.medc[0] = sm.medc[1] = sm.medn[0] = sm.medn[1] = 0;
     }
-#ifdef BC_SMEM_QUEUE
-    if (threadIdx.x < NT / 32) sm.wqn[threadIdx.x] = 0;
-#endif
     int fpass = 0;  // fast-path passes so far (medium-queue counters alternate by parity)
 
     for (;;) {
@@ -1009,10 +1002,6 @@ bc_kernel(KParams p) {
                 f.cnt = &sm.cnt[L % 3];
                 f.kmatch = LV::key(L - 1);
                 f.knew = LV::key(L + 1);
-#ifdef BC_SMEM_QUEUE
-                f.wqn = sm.wqn;
-                f.wq = &sm.wq[0][0];
-#endif
                 const unsigned before = c.scanned;
                 fast_pass<NT, false, true>(p, f, S, lo, hi, L, bigq, sm, c, fpass++ & 1);
                 c.arcs_reached += c.scanned - before;
