@@ -669,6 +669,13 @@ static bcbatch::BParams batch_params(bc_graph *g, const int *d_sources, long lon
     bp.n = g->n;
     bp.ro = g->ro;
     bp.col = g->col;
+    bp.src = g->src;
+    bp.nnz = g->nnz;
+    // multi-source EP levels: Alg. 5 runs (guard ep_min_frontier, only after an EP decision)
+    // and the EP strategy (every level); WE / hybrid batches stay work-efficient
+    bp.ep_guard = g->opt.strategy == BC_STRATEGY_SAMPLING ? g->opt.ep_min_frontier
+                : g->opt.strategy == BC_STRATEGY_EP ? 1 : 0;
+    bp.ep_flag = g->opt.strategy == BC_STRATEGY_SAMPLING ? g->flag : nullptr;
     bp.sources = d_sources;
     bp.perm = g->perm;
     bp.src_base = base;

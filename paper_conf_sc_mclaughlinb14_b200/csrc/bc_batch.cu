@@ -327,6 +327,89 @@ __device__ __forceinline__ void process_range(const BParams &p, const Level &lv,
     if (tprof && lane == 0) tprof[5] += clock64() - tr0;
 }
 
+// ---- one warp's range [a_lo, a_hi) of ALL arcs: a multi-source edge-parallel forward level
+// (Jia et al.'s EP, P:96 / P:112, with one arc scan serving every source of the batch).  The
+// row of arc a is src[a]; a 32-arc window whose rows hold no frontier vertex of any source
+// costs two coalesced loads.  Per arc the same work as process_range<true>: the sigma pull
+// of the row's sources from x = col[a], the discovery of x for the sources that reach it
+// first, x enqueued into Q_{L+1} once (the backward and later WE levels run on the queues).
+__device__ __forceinline__ void process_range_ep(const BParams &p, const Level &lv, int a_lo, int a_hi, Cnt &c,
+                                                 unsigned long long &wor, uint16_t *lst) {
+    const int lane = threadIdx.x & 31;
+    const int L = lv.L;
+    const int LS = p.LS;
+    for (int base = a_lo; base < a_hi; base += 32) {
+        const int a = base + lane;
+        const bool ok = a < a_hi;
+        if (lane == 0) c.sc += (unsigned)min(32, a_hi - base);
+        const int u = ok ? __ldg(&p.src[a]) : 0;
+        const unsigned long long f = ok ? __ldcg(&p.F[(size_t)u * LS + L]) : 0ull;
+        if (!__any_sync(FULL, f != 0ull)) continue;
+        const int x = f ? __ldg(&p.col[a]) : 0;
+        unsigned long long fp = 0ull, fc = 0ull, fn = 0ull;
+        unsigned long long *Fx = p.F + (size_t)x * LS + L;
+        if (f) {
+            if (L > 0) fp = __ldca(Fx - 1);
+            fc = __ldca(Fx);
+            fn = __ldcg(Fx + 1);
+        }
+        const unsigned long long m = f & fp;
+        const unsigned long long dm = f & ~(fp | fc | fn);
+        bool fresh = false;
+        int dv = 0, incl = 0;
+        unsigned long long resv = 0ull;
+        if (dm) {
+            dv = __ldg(&p.ro[x + 1]) - __ldg(&p.ro[x]);
+            const unsigned long long old = atomicOr(Fx + 1, dm);
+            fresh = old == 0ull;
+            unsigned long long nw = dm & ~old;
+            while (nw) {
+                const int b = __ffsll((long long)nw) - 1;
+                nw &= nw - 1ull;
+                p.sig[sidx(p, b, x)] = 0.0;
+                p.dacc[sidx(p, b, x)] = 0.0;
+            }
+        }
+        const unsigned nb = __ballot_sync(FULL, fresh);
+        if (nb) {
+            if (!fresh) dv = 0;
+            incl = dv;
+#pragma unroll
+            for (int s = 1; s < 32; s <<= 1) {
+                const int y = __shfl_up_sync(FULL, incl, s);
+                if (lane >= s) incl += y;
+            }
+            const int tot = __shfl_sync(FULL, incl, 31);
+            if (lane == 0)
+                resv = atomicAdd(&p.qctr[L + 1], ((unsigned long long)__popc(nb) << 40) | (unsigned long long)tot);
+        }
+        c.dag += (unsigned)__popcll(m);
+        if (f) {  // first arc of a frontier row: per-row statistics
+            const int rs = __ldg(&p.ro[u]);
+            if (a == rs) {
+                const unsigned nf = (unsigned)__popcll(f);
+                c.reached += nf;
+                c.ar += nf * (unsigned)(__ldg(&p.ro[u + 1]) - rs);
+                c.dsum += (unsigned long long)L * nf;
+                wor |= f;
+            }
+        }
+        const int npairs = __reduce_add_sync(FULL, (unsigned)__popcll(m));
+        int same = 0;
+        __match_all_sync(FULL, u, &same);
+        if (same && npairs > 96 && __all_sync(FULL, ok)) gather_row_window<true>(p, x, m, u);
+        else if (npairs) accumulate_pairs<true>(p, lst, x, u, m);
+        if (nb) {
+            resv = shfl64(resv, 0);
+            if ((nb >> lane) & 1u) {
+                const int pos = lv.qlo_next + (int)(resv >> 40) + __popc(nb & ((1u << lane) - 1u));
+                p.Q[pos] = x;
+                p.qoff[pos] = (int)(resv & ARC_MASK) + incl - dv;
+            }
+        }
+    }
+}
+
 // delta_b(u) = sigma_b(u) * acc_b(u) for every pair of level L (complete after the
 // barrier that ended backward level L), summed over b into bc[u] (Eq. 3).
 // Thread per (entry, source): 64 consecutive threads share one Q entry.
@@ -377,6 +460,8 @@ __global__ void __launch_bounds__(NT, 768 / NT) batch_kernel(BParams p) {
     cg::grid_group grid = cg::this_grid();
     __shared__ int s_qlo[MAX_LCAP + 4];  // Q offset of each level
     __shared__ int s_A[MAX_LCAP + 4];    // arcs of each level
+    __shared__ unsigned char s_ep[MAX_LCAP + 4];  // forward level L ran edge-parallel
+    const int run_ep = p.ep_flag ? __ldcg(p.ep_flag) : 1;
     __shared__ long long s_ovf;
     __shared__ uint16_t s_lst[NT / 32][32 * BW];  // per-warp (arc, source) pair lists
     uint16_t *lst = s_lst[threadIdx.x >> 5];
@@ -436,11 +521,19 @@ __global__ void __launch_bounds__(NT, 768 / NT) batch_kernel(BParams p) {
                 s_qlo[lv.L + 1] = lv.qlo_next;
                 s_A[lv.L] = lv.A;
             }
+            // multi-source EP level: the union frontier is large enough (Alg. 5 guard)
+            const bool ep = run_ep && p.ep_guard > 0 && lv.qn >= p.ep_guard;
+            if (threadIdx.x == 0) s_ep[lv.L] = ep ? 1 : 0;
             const int nact = lv.A > 0 ? (lv.A + lv.per - 1) / lv.per : 0;
             const long long t0 = clock64();
             long long tp[6] = {0, 0, 0, 0, 0, 0};
             long long *tpp = (p.trace && bt == 0) ? tp : nullptr;
-            if (gw < nact) process_range<true>(p, lv, gw * lv.per, min(lv.A, (gw + 1) * lv.per), cb, wor, lst, tpp);
+            if (ep) {
+                const int per = max(p.min_range, (p.nnz + GW - 1) / GW);
+                if (gw * (long long)per < p.nnz) process_range_ep(p, lv, gw * per, min(p.nnz, (gw + 1) * per), cb, wor, lst);
+            } else if (gw < nact) {
+                process_range<true>(p, lv, gw * lv.per, min(lv.A, (gw + 1) * lv.per), cb, wor, lst, tpp);
+            }
             if (tpp) trace_flush(p, 0, lv.L, tp);
             if (p.trace && bt == 0) trace_level(p, 0, lv.L, lv.A, t0, gw < nact);
             {
@@ -523,17 +616,23 @@ __global__ void __launch_bounds__(NT, 768 / NT) batch_kernel(BParams p) {
         if (blockIdx.x == 0) {
             for (int l = threadIdx.x; l <= Ltop + 1 && l < LS; l += NT) p.qctr[l] = 0ull;
             if (threadIdx.x < 32) {
-                unsigned long long lvs = 0;
+                unsigned long long lvs = 0, lve = 0;
                 for (int l = threadIdx.x; l <= Ltop && l < LS; l += 32) {
-                    lvs += (unsigned long long)__popcll(__ldcg(&p.lvor[l]));
+                    const unsigned long long pc = (unsigned long long)__popcll(__ldcg(&p.lvor[l]));
+                    lvs += pc;
+                    if (s_ep[l]) lve += pc;
                     p.lvor[l] = 0ull;
                 }
 #pragma unroll
-                for (int o = 16; o > 0; o >>= 1) lvs += __shfl_xor_sync(FULL, lvs, o);
+                for (int o = 16; o > 0; o >>= 1) {
+                    lvs += __shfl_xor_sync(FULL, lvs, o);
+                    lve += __shfl_xor_sync(FULL, lve, o);
+                }
                 if (threadIdx.x == 0) {
                     if (!ovf) {
                         atomicAdd(&p.stats->levels, lvs);
-                        atomicAdd(&p.stats->we_levels, lvs);
+                        atomicAdd(&p.stats->we_levels, lvs - lve);
+                        atomicAdd(&p.stats->ep_levels, lve);
                         atomicAdd(&p.stats->sources, (unsigned long long)nb);
                     } else {
                         atomicAdd(&p.stats->batch_overflows, 1ull);

@@ -45,6 +45,12 @@ struct BParams {
     int n;
     const int *__restrict__ ro;   // int32 CSR (internal ids)
     const int *__restrict__ col;
+    const int *__restrict__ src;  // COO source of each arc (multi-source EP levels)
+    int nnz;
+    int ep_guard;                 // a forward level whose union frontier has >= ep_guard vertices
+                                  // is expanded edge-parallel (one scan of all arcs for the 64
+                                  // sources; 0 = never); only when *ep_flag == 1 if ep_flag is set
+    const int *ep_flag;           // Alg. 5 decision (EP run) or nullptr
     const int *sources;           // caller ids; NULL: source = src_base + idx
     const int *perm;              // caller id -> internal id (NULL: identity)
     long long src_base, k;        // this launch's sources: [src_base, src_base + k) of the list

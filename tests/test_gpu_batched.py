@@ -221,3 +221,32 @@ def test_directed_rejected(bcmod):
     with bcmod.BCGraph.from_graph(g, engine="batched") as bg:
         with pytest.raises(bcmod.BCError):
             bg.batch_sources(np.array([0], dtype=np.int32))
+
+
+@pytest.mark.parametrize("key,k,strategy", [("c1", None, "ep"), ("c1", 600, "sampling"), ("c4", 200, "ep"),
+                                            ("c4", 700, "sampling"), ("c5k", 640, "sampling")])
+def test_multi_source_ep_levels(bcmod, oracle_mod, key, k, strategy):
+    """Multi-source edge-parallel levels: one scan of all arcs serves the
+    64 sources of a batch when the union frontier reaches the Alg. 5 guard (strategy
+    sampling, after an EP decision) or on every level (strategy ep).  BC, the per-source
+    d / sigma / delta of a batch and the byte-model counters equal the oracle's."""
+    g = graph(key)
+    src = None if k is None else gg.CONFIGS[key].sources(g)[:k] if gg.CONFIGS[key].k \
+        else gg.sample_sources(g, k, seed=13)
+    with bcmod.BCGraph.from_graph(g, engine="batched", strategy=strategy) as bg:
+        check_bc(bg, g, src, oracle_mod, nthreads=16)
+        st = bg.stats()
+        assert st["ep_levels"] > 0 and st["batches"] > 0
+        if strategy == "ep":
+            assert st["we_levels"] == 0
+        else:
+            assert st["sampling_ep"] == 1
+        sub = (np.arange(g.n, dtype=np.int32) if src is None else src)[:40]
+        check_batch(bg, g, sub, oracle_mod)   # the last call's Alg. 5 decision stands (EP)
+    if key != "c5k":
+        refs = [oracle_mod.single_source(g, int(s)) for s in (np.arange(g.n) if src is None else src)]
+        assert st["n_reached"] == sum(r["n_reached"] for r in refs)
+        assert st["arcs_reached"] == sum(r["arcs_reached"] for r in refs)
+        assert st["dag_arcs"] == sum(r["dag_arcs"] for r in refs)
+        assert st["levels"] == sum(r["num_levels"] for r in refs)
+        assert st["dist_sum"] == sum(int(r["d"][r["d"] >= 0].sum()) for r in refs)

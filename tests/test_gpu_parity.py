@@ -503,3 +503,30 @@ def test_optimistic_we_with_handover(bcmod, oracle_mod, key, strategy, expect_ha
             for s in src[:3]:
                 ref = oracle_mod.single_source(g, int(s))
                 assert bg.single_source(int(s))["level_modes"].tolist() == sel.hybrid_modes(ref["level_sizes"].tolist())
+
+
+@pytest.mark.parametrize("key,strategy,k,inflight,extra", [
+    ("c1", "sampling", 700, 0, {}),                      # paper parameters: some sources hand over
+    ("c1", "hybrid", 300, 1, {"alpha": 0, "beta": 16}),  # one CTA; EP from the first big change
+    ("c4", "hybrid", 120, 5, {}),
+])
+def test_handover_counters_and_duplicates(bcmod, oracle_mod, key, strategy, k, inflight, extra):
+    """A handed-over source is counted once: its partial forward on the WE-only kernel is
+    rolled back (levels, distance sum, arcs, DAG arcs) and recomputed by the EP-capable
+    kernel.  The byte-model counters and the level count then equal the oracle's, and BC
+    is the oracle's -- also with duplicate sources and a single CTA in flight."""
+    g = graph(key)
+    src = gg.sample_sources(g, k, seed=21) if key == "c1" else gg.CONFIGS[key].sources(g)[:k]
+    src = np.concatenate([src, src[:7]])      # duplicates count with multiplicity (R15)
+    opts = dict(strategy=strategy, inflight=inflight, **extra)
+    with bcmod.BCGraph.from_graph(g, **opts) as bg:
+        check_bc(bg, g, src, oracle_mod)
+        st = bg.stats()
+    assert st["handovers"] > 0
+    refs = [oracle_mod.single_source(g, int(s)) for s in src]
+    assert st["sources"] == src.size
+    assert st["n_reached"] == sum(r["n_reached"] for r in refs)
+    assert st["arcs_reached"] == sum(r["arcs_reached"] for r in refs)
+    assert st["dag_arcs"] == sum(r["dag_arcs"] for r in refs)
+    assert st["levels"] == sum(r["num_levels"] for r in refs)
+    assert st["dist_sum"] == sum(int(r["d"][r["d"] >= 0].sum()) for r in refs)
