@@ -158,6 +158,12 @@ typedef struct bc_stats {
     int64_t handovers;        /* Alg. 4 / Alg. 5 runs on the fast work-efficient kernel: sources
                                  whose selector picked an EP level and were therefore re-run
                                  from scratch by the EP-capable kernel (0 if none)             */
+    int64_t group_wait_cycles; /* group engine: SM cycles its CTAs spent waiting at the per-level
+                                 group barriers after finishing their own share (summed over
+                                 CTAs; load-imbalance + barrier latency), 0 on other engines  */
+    int32_t group_mode;       /* group engine level passes of the last call: 0 generic row_pass,
+                                 1 fast path, 2 thin rows (bc_thin.cuh); -1 not run           */
+    int32_t pad2_;
 } bc_stats;
 
 /* Copy a CSR graph to `device` and allocate the per-source workspace.

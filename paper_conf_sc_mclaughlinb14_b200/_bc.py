@@ -52,7 +52,8 @@ class bc_stats(ctypes.Structure):
                 ("kernel_ms", ctypes.c_double), ("phase_cycles", ctypes.c_int64 * 4),
                 ("batches", ctypes.c_int64), ("batch_overflows", ctypes.c_int64),
                 ("engines", ctypes.c_int32), ("pad_", ctypes.c_int32), ("dist_sum", ctypes.c_int64),
-                ("handovers", ctypes.c_int64)]
+                ("handovers", ctypes.c_int64), ("group_wait_cycles", ctypes.c_int64),
+                ("group_mode", ctypes.c_int32), ("pad2_", ctypes.c_int32)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_}

@@ -113,6 +113,7 @@ struct bc_graph {
     int code_words = 0, fb_words = 0;
     int seq_max_deg = 32;
     int max_deg = 0;      // largest out-degree of the graph
+    int thin_wide = 0;    // rows longer than bcgroup::THIN_MAX_ROW
     int warp_max_deg = 4096;
     // graph
     char *graph_buf = nullptr;          // ro | col | src
@@ -485,16 +486,30 @@ static int group_count(const bc_graph *g, int grid) {
 
 // The group engine's work-efficient levels run through the fast path on degree-relabelled
 // (skewed) graphs and through the generic row_pass otherwise (measured).
-static bool group_fast(const bc_graph *g) {
-    if (const char *e = getenv("BC_GROUP_FAST")) return atoi(e) != 0;  // tuning override
-    return g->perm != nullptr;
+// Thin rows (bc_thin.cuh) need the successor bitmap and a per-CTA queue (bigq, stride_big
+// entries) that holds every row longer than THIN_MAX_ROW.
+static bool thin_ok(const bc_graph *g) {
+    return g->opt.succ_bits >= 0 && (size_t)g->thin_wide + 2 <= g->stride_big;
+}
+
+static int group_mode(const bc_graph *g) {
+    int m = -1;
+    if (const char *e = getenv("BC_GROUP_MODE")) m = atoi(e);  // tuning override
+    else if (const char *e = getenv("BC_GROUP_FAST")) m = atoi(e) != 0 ? bcgroup::GM_FAST : bcgroup::GM_GENERIC;
+    // auto (B200, c5ws 2,048 sources, kernel ms): degree-relabelled graphs take the fast path
+    // (c5k 1959 against 2104 generic, 4036+ thin); graphs in their own order with >= 2^21
+    // vertices take thin rows (c5ws 1416 against 1503 generic, 1548 fast), smaller ones the
+    // generic row_pass (CSR-order sums)
+    if (m < 0) m = g->perm ? bcgroup::GM_FAST : (g->n >= (1 << 21) ? bcgroup::GM_THIN : bcgroup::GM_GENERIC);
+    if (m == bcgroup::GM_THIN && !thin_ok(g)) m = bcgroup::GM_GENERIC;
+    return m;
 }
 
 static int alloc_group(bc_graph *g) {
     bc_graph::Group &q = g->gr;
     const int nt = g->n >= (1 << 17) ? 512 : 256;
     int per_sm = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bcgroup::group_kernel_fn(nt, group_fast(g)), nt, 0));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bcgroup::group_kernel_fn(nt, group_mode(g)), nt, 0));
     if (per_sm < 1) return fail(BC_EINTERNAL, "group kernel cannot be resident");
     const int grid = per_sm * g->num_sms;
     const int G = group_count(g, grid);
@@ -596,7 +611,7 @@ static int launch_group(bc_graph *g, const KParams &p0, cudaStream_t st) {
     }
     lc.attrs = attr;
     lc.numAttrs = na;
-    CK(cudaLaunchKernelExC(&lc, bcgroup::group_kernel_fn(q.nt, group_fast(g)), args));
+    CK(cudaLaunchKernelExC(&lc, bcgroup::group_kernel_fn(q.nt, group_mode(g)), args));
     CK(cudaGetLastError());
     g->launches++;
     g->bc_launches++;
@@ -775,7 +790,10 @@ static int create_impl(bc_graph *g, const int64_t *ro64, const int32_t *col_in) 
         for (int v = 0; v <= n; ++v) ro32[v] = (int)ro64[v];
     }
     g->h_ro = ro32;
-    for (int v = 0; v < n; ++v) g->max_deg = std::max(g->max_deg, ro32[v + 1] - ro32[v]);
+    for (int v = 0; v < n; ++v) {
+        g->max_deg = std::max(g->max_deg, ro32[v + 1] - ro32[v]);
+        if (ro32[v + 1] - ro32[v] > bcgroup::THIN_MAX_ROW) g->thin_wide++;
+    }
     CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
     CK(cudaEventCreateWithFlags(&g->done, cudaEventDisableTiming));
     for (auto &e : g->tev) CK(cudaEventCreate(&e));
@@ -1444,6 +1462,9 @@ extern "C" int bc_get_stats(bc_graph *g, bc_stats *st) {
     st->pad_ = 0;
     st->dist_sum = (int64_t)h.dist_sum;
     st->handovers = 0;
+    st->group_wait_cycles = (int64_t)h.group_wait;
+    st->group_mode = (g->engines & 4) ? group_mode(g) : -1;
+    st->pad2_ = 0;
     if (g->fb_used) {
         unsigned long long fb = 0;
         CK(cudaMemcpy(&fb, g->fb_n, sizeof(fb), cudaMemcpyDeviceToHost));

@@ -171,7 +171,7 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
             if (pos + 4 > end) valid &= 0xFu >> min(4, pos + 4 - end);
             const unsigned sbits = (unsigned)(win >> off) & valid;
             if (!sbits) continue;
-            const int4 c4 = *reinterpret_cast<const int4 *>(cols + pos);
+            const int4 c4 = ld_col4(cols + pos);
             const int u[4] = {c4.x, c4.y, c4.z, c4.w};
             double g[4];
 #pragma unroll
@@ -182,14 +182,14 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
         return acc;
     }
     int4 nx = make_int4(0, 0, 0, 0);
-    if (nq > 0) nx = *reinterpret_cast<const int4 *>(cols + q0);
+    if (nq > 0) nx = ld_col4(cols + q0);
     unsigned dag = 0;
     int w0 = beg >> 5;
     uint64_t win = 0;
     for (int q = 0; q < maxq; ++q) {
         const int pos = q0 + 4 * q;
         const int4 c4 = nx;
-        if (q + 1 < nq) nx = *reinterpret_cast<const int4 *>(cols + pos + 4);
+        if (q + 1 < nq) nx = ld_col4(cols + pos + 4);
         unsigned valid = q < nq ? 0xFu : 0u;
         if (pos < beg) valid &= 0xFu << (beg - pos);
         if (pos + 4 > end) valid &= 0xFu >> min(4, pos + 4 - end);
@@ -276,7 +276,7 @@ __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *_
             if (!__any_sync(FULL, s[0] | s[1] | s[2] | s[3])) continue;
             int u[4];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) u[j] = s[j] ? cols[a[j]] : 0;
+            for (int j = 0; j < 4; ++j) u[j] = s[j] ? ld_col(cols + a[j]) : 0;
             double g[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) g[j] = ldca_if(f.sig + u[j], s[j]);
@@ -288,7 +288,7 @@ __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *_
     unsigned dag = 0;
     int un_[4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) un_[j] = b + t + j * stride < e ? cols[b + t + j * stride] : 0;
+    for (int j = 0; j < 4; ++j) un_[j] = b + t + j * stride < e ? ld_col(cols + b + t + j * stride) : 0;
     // each step's gathers are added one step late, after the next step's gathers are issued
     // (same order of additions, so the same sums; B200: c4 160.3 -> 157.3 ms per 4,096
     // sources, c5k group 1960 -> 1947 ms per 2,048)
@@ -304,7 +304,7 @@ __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *_
         const int bn = base + 4 * stride;
         if (bn < e) {
 #pragma unroll
-            for (int j = 0; j < 4; ++j) un_[j] = bn + t + j * stride < e ? cols[bn + t + j * stride] : 0;
+            for (int j = 0; j < 4; ++j) un_[j] = bn + t + j * stride < e ? ld_col(cols + bn + t + j * stride) : 0;
         }
         int k[4];
 #pragma unroll

@@ -7,6 +7,7 @@
 #define BC_INSTANCE_TU
 #include "bc_kernels.cuh"
 #include "bc_group.cuh"
+#include "bc_thin.cuh"
 
 namespace bcgroup {
 
@@ -22,15 +23,19 @@ __device__ __forceinline__ unsigned long long ld_acquire(const unsigned long lon
 // before the arrival publishes the CTA's writes; the acquire load / fence after it
 // invalidate this SM's L1 (CCTL.IVALL), so plain loads after the barrier see every write
 // made before it.
-__device__ __forceinline__ void group_sync(unsigned long long *bar, unsigned long long &target, int C) {
+// `wait` (thread 0) accumulates the cycles from this CTA's arrival to the release.
+__device__ __forceinline__ void group_sync(unsigned long long *bar, unsigned long long &target, int C,
+                                           unsigned long long *wait) {
     __syncthreads();
     if (threadIdx.x == 0) {
+        const long long t0 = clock64();
         target += (unsigned long long)C;
         __threadfence();
         atomicAdd(bar, 1ull);
         while (ld_acquire(bar) < target) {
         }
         __threadfence();
+        *wait += (unsigned long long)(clock64() - t0);
     }
     __syncthreads();
 }
@@ -128,8 +133,15 @@ __device__ __forceinline__ int group_compact(uint32_t *nb, int words, int r, int
 // generic row_pass.  Measured per graph kind on B200: faster on the skewed,
 // degree-relabelled Kronecker graph (c5k 2100 -> 2024 ms per 2,048 sources; 1954 with 18
 // CTAs per group), slower on the unskewed small world (c5ws 1500 -> 1568 ms, the backward).
-template <int NT, bool FASTG>
-__global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p, GParams gp) {
+// MODE: GM_GENERIC (row_pass), GM_FAST (bc_fast.cuh), GM_THIN (bc_thin.cuh, virtual warps).
+#ifndef BC_THIN_MINB
+#define BC_THIN_MINB 2
+#endif
+template <int NT, int MODE>
+__global__ void __launch_bounds__(NT, NT >= 512 ? (MODE == GM_THIN ? BC_THIN_MINB : 2) : 4)
+group_kernel(KParams p, GParams gp) {
+    constexpr bool FASTG = MODE == GM_FAST;
+    constexpr bool THIN = MODE == GM_THIN;
     constexpr int NW = NT / 32;
     __shared__ Smem<NT> sm;
     __shared__ int2 s_reg[RCAP];  // this CTA's share of level L in S: (offset, count), L < RCAP
@@ -177,9 +189,22 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
         f.knew = knew;
         return f;
     };
+    auto tl_ = [&](uint32_t *gnb, int kmatch, int knew) {
+        ThinLevel t;
+        t.ro = p.ro;
+        t.col = p.col;
+        t.sbr = sb;
+        t.codes = lv.w;
+        t.nb = gnb;
+        t.sb = sb;
+        t.sig = sigma;
+        t.kmatch = kmatch;
+        t.knew = knew;
+        return t;
+    };
     const long long K = p.k;
     if (r == 0 && tid == 0) *next_idx = (long long)atomicAdd(p.work_counter, 1ULL);
-    group_sync(bar, target, C);
+    group_sync(bar, target, C, &sm.st.gwait);
 
     for (;;) {
         const long long idx = *(volatile long long *)next_idx;
@@ -197,6 +222,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             lvl[0] = 1;
             lvl[1] = 0;
         }
+        if constexpr (THIN) __syncthreads();   // Alg. 1 stores above, read by other lanes below
         int mylo = 0, mycnt = r == 0 ? 1 : 0;  // this CTA's vertices of level L: S[mylo, +mycnt)
         if (tid == 0) s_reg[0] = make_int2(mylo, mycnt);
         int prevlo = 0, prevcnt = 0;
@@ -207,7 +233,10 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             uint32_t *nbw_next = nbb + (size_t)((L + 1) % 3) * nbw;
             // (a) Alg. 2 over this CTA's share of level L (ends with a CTA barrier)
             if (mycnt > 0) {
-                if constexpr (!FASTG) {
+                if constexpr (THIN) {
+                    thin_pass<NT, true>(p, tl_(nbw_next, GlobalCodes::key(L - 1), GlobalCodes::key(L + 1)), S, mylo,
+                                        mylo + mycnt, L, bigq, sm, c);
+                } else if constexpr (!FASTG) {
                     forward_we<false, NT, GlobalCodes, true>(p, lv, sigma, S, bigq, nbw_next, sb, L, mylo,
                                                              mylo + mycnt, sm, c);
                 } else {
@@ -218,7 +247,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
                 }
             }
             // (b) level L+1 is complete once every CTA got here
-            group_sync(bar, target, C);
+            group_sync(bar, target, C, &sm.st.gwait);
             const int tot = *(volatile int *)&lvl[L & 3];
             if (r == 0 && tid == 0 && p.dbg_fcyc && L > 0 && L - 1 < p.dbg_max_levels) {
                 const long long now = clock64();
@@ -261,7 +290,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
                     p.dbg_sigma[v] = __ldcg(&sigma[v]);
                 }
             }
-            group_sync(bar, target, C);
+            group_sync(bar, target, C, &sm.st.gwait);
         }
         // Stage 2 (Alg. 3).  Deepest level: delta = 0, omega = 1/sigma (in place), by owner.
         if (maxdepth >= 1) {
@@ -269,7 +298,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
                 const int v = S[i];
                 sigma[v] = 1.0 / __ldcg(&sigma[v]);
             }
-            group_sync(bar, target, C);
+            group_sync(bar, target, C, &sm.st.gwait);
         }
         // Backward levels: each CTA finishes the vertices it expanded in the forward (same
         // ownership, same locality); levels >= RCAP in 32-vertex chunks over the group.
@@ -277,7 +306,10 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             const long long t0 = clock64();
             if (Lb < RCAP) {
                 const int2 rg = s_reg[Lb];
-                if constexpr (!FASTG) {
+                if constexpr (THIN) {
+                    thin_pass<NT, false>(p, tl_(nullptr, GlobalCodes::key(Lb + 1), 0), S, rg.x, rg.x + rg.y, Lb, bigq,
+                                         sm, c);
+                } else if constexpr (!FASTG) {
                     backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, rg.x, rg.x + rg.y, sm, c);
                 } else {
                     fast_pass<NT, true, false>(p, mk(nullptr, GlobalCodes::key(Lb + 1), 0), S, rg.x, rg.x + rg.y, Lb,
@@ -289,7 +321,10 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
                     sm.gwn = C * NW;
                 }
                 __syncthreads();
-                if constexpr (!FASTG) {
+                if constexpr (THIN) {
+                    thin_pass<NT, false>(p, tl_(nullptr, GlobalCodes::key(Lb + 1), 0), S, ends[Lb], ends[Lb + 1], Lb,
+                                         bigq, sm, c);
+                } else if constexpr (!FASTG) {
                     backward_we<NT, GlobalCodes, true>(p, lv, sigma, S, bigq, sb, Lb, ends[Lb], ends[Lb + 1], sm, c);
                 } else {
                     fast_pass<NT, true, false>(p, mk(nullptr, GlobalCodes::key(Lb + 1), 0), S, ends[Lb], ends[Lb + 1],
@@ -301,7 +336,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
                     sm.gwn = NW;
                 }
             }
-            group_sync(bar, target, C);
+            group_sync(bar, target, C, &sm.st.gwait);
             if (r == 0 && tid == 0 && p.dbg_bcyc && Lb < p.dbg_max_levels) p.dbg_bcyc[Lb] = clock64() - t0;
         }
         // Reset of this source's codes and successor bits (the bitmaps are clear already),
@@ -331,7 +366,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             sm.st.reached += (unsigned long long)S_len;
             *next_idx = (long long)atomicAdd(p.work_counter, 1ULL);
         }
-        group_sync(bar, target, C);
+        group_sync(bar, target, C, &sm.st.gwait);
     }
 
     if (tid == 0) {
@@ -345,6 +380,7 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
             atomicAdd(&gs->phase_cycles[0], sm.st.cyc[0]);
             atomicAdd(&gs->phase_cycles[2], sm.st.cyc[2]);
         }
+        atomicAdd(&gs->group_wait, sm.st.gwait);
         atomicAdd(&gs->arcs_reached, sm.st.ar);
         atomicAdd(&gs->dag_arcs, sm.st.dg);
         atomicAdd(&gs->arcs_scanned, sm.st.sc);
@@ -352,9 +388,10 @@ __global__ void __launch_bounds__(NT, NT >= 512 ? 2 : 4) group_kernel(KParams p,
     }
 }
 
-const void *group_kernel_fn(int nt, bool fast) {
-    if (fast) return nt == 256 ? (const void *)group_kernel<256, true> : (const void *)group_kernel<512, true>;
-    return nt == 256 ? (const void *)group_kernel<256, false> : (const void *)group_kernel<512, false>;
+const void *group_kernel_fn(int nt, int mode) {
+    if (mode == GM_FAST) return nt == 256 ? (const void *)group_kernel<256, GM_FAST> : (const void *)group_kernel<512, GM_FAST>;
+    if (mode == GM_THIN) return nt == 256 ? (const void *)group_kernel<256, GM_THIN> : (const void *)group_kernel<512, GM_THIN>;
+    return nt == 256 ? (const void *)group_kernel<256, GM_GENERIC> : (const void *)group_kernel<512, GM_GENERIC>;
 }
 
 }  // namespace bcgroup

@@ -41,10 +41,15 @@ struct GParams {
     int own_block;               // bitmap words per ownership block (>= 1), see Owned
 };
 
+// Level passes of the group kernel: generic row_pass, the fast path (bc_fast.cuh, degree-
+// relabelled graphs) or thin rows on virtual warps (bc_thin.cuh, graphs without hubs).
+enum : int { GM_GENERIC = 0, GM_FAST = 1, GM_THIN = 2 };
+constexpr int THIN_MAX_ROW = 32;  // GM_THIN: longer rows are queued (<= stride_big per CTA), one warp each
+
 // Kernel symbol for a block size (256 or 512 threads); launched cooperatively with
 // arguments (KParams, GParams).  KParams: sigma / S / ends / gcodes / nbits (3 buffers of
 // nb_words) / sbits are per GROUP (strides stride_n, stride_e, stride_codes, stride_nb,
 // stride_sb); bigq is per CTA (stride_big).
-const void *group_kernel_fn(int nt, bool fast);
+const void *group_kernel_fn(int nt, int mode);
 
 }  // namespace bcgroup

@@ -51,6 +51,7 @@ struct DevStats {
     int pad;
     unsigned long long batches, batch_overflows;  // multi-source engine (bc_batch.cu)
     unsigned long long dist_sum;  // sum over sources of sum_t d(s,t) over reached t (self-check)
+    unsigned long long group_wait;  // group engine: CTA cycles waiting at group barriers
 };
 
 struct KParams {
@@ -134,6 +135,7 @@ struct CtaStats {
     unsigned long long lv[2];   // levels expanded WE / EP
     unsigned long long cyc[4];  // fwd WE, fwd EP, bwd WE, bwd EP
     unsigned long long dsum;    // sum of d(s,t) over the reached t of this CTA's sources
+    unsigned long long gwait;   // group engine: cycles waiting at group barriers (thread 0)
     int inexact;
 };
 
@@ -310,6 +312,13 @@ __device__ __forceinline__ double warp_sum(double v) {
     return v;
 }
 
+
+// Column loads of the CSR.  (An L2 evict-first / L1 no-allocate hint on them was measured
+// slower on B200: c4 159 -> 178 ms per 4,096 sources, c5ws 1500 -> 1715, c5k 1956 -> 2212 ms
+// per 2,048 -- neighbouring rows share L1 lines and concurrent sources share L2 lines.)
+__device__ __forceinline__ int4 ld_col4(const int *p) { return *reinterpret_cast<const int4 *>(p); }
+__device__ __forceinline__ int ld_col(const int *p) { return *p; }
+
 #ifndef BC_UNROLL
 #define BC_UNROLL 4
 #endif
@@ -349,7 +358,7 @@ __device__ __forceinline__ double coop_sum(const int *__restrict__ cols, int b, 
                 ok[j] = a < e && ((__ldcg(&ab.sb[a >> 5]) >> (a & 31)) & 1u);
             }
 #pragma unroll
-            for (int j = 0; j < U; ++j) u[j] = ok[j] ? cols[base + t + j * stride] : 0;
+            for (int j = 0; j < U; ++j) u[j] = ok[j] ? ld_col(cols + base + t + j * stride) : 0;
 #pragma unroll
             for (int j = 0; j < U; ++j) g[j] = ok[j] ? gather(u[j], ab.knext) : 0.0;
 #pragma unroll
@@ -359,7 +368,7 @@ __device__ __forceinline__ double coop_sum(const int *__restrict__ cols, int b, 
     }
     int un[U];
 #pragma unroll
-    for (int j = 0; j < U; ++j) un[j] = b + t + j * stride < e ? cols[b + t + j * stride] : 0;
+    for (int j = 0; j < U; ++j) un[j] = b + t + j * stride < e ? ld_col(cols + b + t + j * stride) : 0;
     for (int base = b; base < e; base += U * stride) {
         int u[U], k[U];
         bool ok[U];
@@ -372,7 +381,7 @@ __device__ __forceinline__ double coop_sum(const int *__restrict__ cols, int b, 
         const int bn = base + U * stride;
         if (bn < e) {
 #pragma unroll
-            for (int j = 0; j < U; ++j) un[j] = bn + t + j * stride < e ? cols[bn + t + j * stride] : 0;
+            for (int j = 0; j < U; ++j) un[j] = bn + t + j * stride < e ? ld_col(cols + bn + t + j * stride) : 0;
         }
 #pragma unroll
         for (int j = 0; j < U; ++j) k[j] = probe(u[j]);
@@ -441,7 +450,7 @@ __device__ __forceinline__ double seq_row_bits(const int *__restrict__ cols, int
         if (ab.mode == 2) {
             const unsigned bits = (unsigned)(win >> off) & valid;
             if (!bits) continue;
-            const int4 c4 = *reinterpret_cast<const int4 *>(cols + q);
+            const int4 c4 = ld_col4(cols + q);
             const int u[4] = {c4.x, c4.y, c4.z, c4.w};
             double g[4];
 #pragma unroll
@@ -450,7 +459,7 @@ __device__ __forceinline__ double seq_row_bits(const int *__restrict__ cols, int
             for (int j = 0; j < 4; ++j) acc += g[j];
             continue;
         }
-        const int4 c4 = *reinterpret_cast<const int4 *>(cols + q);
+        const int4 c4 = ld_col4(cols + q);
         int u[4] = {c4.x, c4.y, c4.z, c4.w}, k[4];
         bool ok[4];
         double g[4];
@@ -495,10 +504,10 @@ __device__ __forceinline__ double seq_row(const int *__restrict__ cols, int a, i
     double acc = 0.0;
     int q = a & ~3;
     if (q >= e) return acc;
-    int4 nx = *reinterpret_cast<const int4 *>(cols + q);
+    int4 nx = ld_col4(cols + q);
     for (; q < e; q += 4) {
         const int4 c4 = nx;
-        if (q + 4 < e) nx = *reinterpret_cast<const int4 *>(cols + q + 4);
+        if (q + 4 < e) nx = ld_col4(cols + q + 4);
         unsigned valid = 0xFu;
         if (q < a) valid &= 0xFu << (a - q);
         if (q + 4 > e) valid &= 0xFu >> (q + 4 - e);

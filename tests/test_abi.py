@@ -60,6 +60,7 @@ int main(void){
          offsetof(bc_stats, kernel_ms));
   printf("%zu %zu %d\n", offsetof(bc_options, engine), offsetof(bc_options, group_ctas), BC_ENGINE_GROUP);
   printf("%zu %zu\n", offsetof(bc_stats, dist_sum), offsetof(bc_stats, handovers));
+  printf("%zu %zu\n", offsetof(bc_stats, group_wait_cycles), offsetof(bc_stats, group_mode));
   return 0; }
 """
     import tempfile
@@ -72,7 +73,8 @@ int main(void){
     O, S = _bc.bc_options, _bc.bc_stats
     assert vals == [ctypes.sizeof(O), O.gamma.offset, O.level_store.offset, ctypes.sizeof(S),
                     S.sampling_ep.offset, S.inflight.offset, S.kernel_ms.offset,
-                    O.engine.offset, O.group_ctas.offset, _bc.ENGINES["group"], S.dist_sum.offset, S.handovers.offset]
+                    O.engine.offset, O.group_ctas.offset, _bc.ENGINES["group"], S.dist_sum.offset, S.handovers.offset,
+                    S.group_wait_cycles.offset, S.group_mode.offset]
 
 
 def test_default_options_are_the_papers(lib):

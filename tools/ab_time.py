@@ -67,7 +67,9 @@ def main():
         print(json.dumps({"tag": a.tag, "config": key, "sources": int(src.size), "opts": opts,
                           "kernel_ms": statistics.median(ms), "all_ms": ms, "gteps": gteps,
                           "engines": st["engines"], "phase_cycles": st["phase_cycles"], "levels": st["levels"],
-                          "arcs_scanned": st["arcs_scanned"], "file": name}), flush=True)
+                          "arcs_scanned": st["arcs_scanned"], "group_wait_cycles": st.get("group_wait_cycles", 0),
+                          "group_mode": st.get("group_mode", -1), "inflight": st["inflight"],
+                          "file": name}), flush=True)
 
 
 if __name__ == "__main__":
