@@ -114,6 +114,7 @@ struct bc_graph {
     int seq_max_deg = 32;
     int max_deg = 0;      // largest out-degree of the graph
     int thin_wide = 0;    // rows longer than bcgroup::THIN_MAX_ROW
+    int bpush = 2;        // fast path backward push ratio (KParams::bpush; BC_BPUSH overrides)
     int warp_max_deg = 4096;
     // graph
     char *graph_buf = nullptr;          // ro | col | src
@@ -176,6 +177,7 @@ struct bc_graph {
         int ready = 0, failed = 0, nt = 512, grid = 0, G = 0, code_words = 0, sb = 0;
         unsigned long long *ctl = nullptr;
         double *sigma = nullptr;
+        double *acc = nullptr;  // backward push accumulators (fast path), zero between uses
         int *S = nullptr, *ends = nullptr, *bigq = nullptr;
         uint32_t *codes = nullptr, *nb = nullptr, *sbits = nullptr;
     } gr;
@@ -462,6 +464,7 @@ static void free_group(bc_graph *g) {
     bc_graph::Group &q = g->gr;
     cudaFree(q.ctl);
     cudaFree(q.sigma);
+    cudaFree(q.acc);
     cudaFree(q.S);
     cudaFree(q.ends);
     cudaFree(q.bigq);
@@ -536,6 +539,10 @@ static int alloc_group(bc_graph *g) {
         CK(cudaMemset(q.sbits, 0, ng * (size_t)g->sb_words * 4));
     }
     CK(cudaMemset(q.sigma, 0, ng * g->stride_n * sizeof(double)));
+    if (group_mode(g) == bcgroup::GM_FAST) {
+        CK(cudaMalloc(&q.acc, ng * g->stride_n * sizeof(double)));
+        CK(cudaMemset(q.acc, 0, ng * g->stride_n * sizeof(double)));
+    }
     CK(cudaDeviceSynchronize());
     q.ready = 1;
     return BC_OK;
@@ -575,6 +582,8 @@ static int launch_group(bc_graph *g, const KParams &p0, cudaStream_t st) {
     const bc_graph::Group &q = g->gr;
     KParams p = p0;
     p.sigma = q.sigma;
+    p.omega = q.acc;  // push accumulators (nullptr: the backward always pulls)
+    if (!q.acc) p.bpush = 0;
     p.S = q.S;
     p.ends = q.ends;
     p.bigq = q.bigq;
@@ -973,6 +982,8 @@ static KParams base_params(bc_graph *g, double *d_bc) {
     p.sb_words = g->sb_words;
     p.seq_max_deg = g->seq_max_deg;
     p.medq = g->max_deg > g->seq_max_deg ? 1 : 0;
+    p.bpush = g->bpush;
+    if (const char *e = getenv("BC_BPUSH")) p.bpush = std::max(0, atoi(e));  // tuning override
     p.warp_max_deg = g->warp_max_deg;
     p.stats = g->stats;
     p.sampled_flag = g->flag;

@@ -394,6 +394,10 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
             deg = rows[v + 1] - beg;
         }
         c.scanned += deg;
+        if (FWD && p.bpush && L < NLEV_ARCS) {  // arcs of level L's rows (backward push choice)
+            const unsigned a = __reduce_add_sync(FULL, (unsigned)deg);
+            if (lane == 0 && a) atomicAdd(&sm.alev[L], a);
+        }
         const bool seq = v >= 0 && deg <= seq_max;
         double sw = 0.0;
         if (!FWD && seq) sw = __ldcg(&f.sig[v]);  // sigma[w], issued early
@@ -475,6 +479,102 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
             __syncthreads();
         }
     }
+}
+
+__device__ __forceinline__ void red_add_f64_if(double *addr, double val, bool c) {
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q red.global.add.f64 [%0], %1;\n\t}"
+                 :
+                 : "l"(addr), "d"(val), "r"((unsigned)c)
+                 : "memory");
+}
+
+// Backward level L finished by PUSHING (the dependency sum of Alg. 3 l.5-9, P:202-227,
+// accumulated from the other side of each DAG arc, with atomics as the paper notes an
+// edge-parallel backward needs): every level-(L+1) vertex w adds omega[w] to
+// acc[v] of each predecessor v (code key(L), a shared-memory probe), then every level-L
+// vertex finishes from acc: delta = sigma * acc, omega = (1 + delta) / sigma, bc += delta
+// (Eq. 3).  Scans A_{L+1} arcs instead of A_L: on Kronecker graphs the big middle level's
+// rows hold most arcs, the level below it few.  The sums are the same up to order (fp64
+// atomics; checked at 1e-9).  S[lo, hi) = level L, S[hi, hi2) = level L+1.  Ends with a
+// barrier.
+// Pushes of the rows S[lo2, hi2) (level L+1) by warps gw0 + wid of gwn; G: global codes.
+template <int NT, bool G>
+__device__ __forceinline__ void push_rows(const KParams &p, const uint32_t *sw, const double *sig_om, double *acc,
+                                          const int *__restrict__ S, int lo2, int hi2, int kpred, int gw0, int gwn,
+                                          Counters &c) {
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int *__restrict__ rows = p.ro;
+    const int *__restrict__ cols = p.col;
+    auto code = [&](int u) -> int {
+        if (!G) return code_at(sw, u);
+        const uint32_t wd = __ldca(&sw[(unsigned)u >> 4]);  // codes are final in the backward
+        return (int)(__funnelshift_r(wd, wd, (unsigned)u << 1) & 3u);
+    };
+    for (int base = lo2 + (gw0 + wid) * 32; base < hi2; base += gwn * 32) {
+        const int i = base + lane;
+        int v = -1, beg = 0, end = 0;
+        double om = 0.0;
+        if (i < hi2) {
+            v = S[i];
+            beg = rows[v];
+            end = rows[v + 1];
+            om = __ldcg(&sig_om[v]);  // omega[w] (level L+1 is finished)
+        }
+        c.scanned += end - beg;
+        const bool one = end - beg <= 32;
+        const int e1 = one ? end : beg;
+        const int nq = (e1 - beg + 3) >> 2;
+        const int maxq = (int)__reduce_max_sync(FULL, (unsigned)nq);
+        for (int q = 0; q < maxq; ++q) {
+            int u[4];
+            bool ok[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const int a = beg + 4 * q + j;
+                ok[j] = a < e1;
+                u[j] = ok[j] ? ld_col(cols + a) : 0;
+            }
+#pragma unroll
+            for (int j = 0; j < 4; ++j) red_add_f64_if(acc + u[j], om, ok[j] && code(u[j]) == kpred);
+        }
+        unsigned wide = __ballot_sync(FULL, v >= 0 && !one);
+        while (wide) {  // longer rows: the whole warp, 32 arcs per step
+            const int ld = __ffs(wide) - 1;
+            wide &= wide - 1u;
+            const int b = __shfl_sync(FULL, beg, ld), e = __shfl_sync(FULL, end, ld);
+            const double w = __shfl_sync(FULL, om, ld);
+            for (int a = b + lane; a < e; a += 32) {
+                const int u = ld_col(cols + a);
+                red_add_f64_if(acc + u, w, code(u) == kpred);
+            }
+        }
+    }
+}
+
+// Finish of the level-L vertices S[lo, hi) from their pushed sums (acc zeroed after use
+// when ZERO, so the array is clean for the next pushed level).
+template <int NT, bool ZERO>
+__device__ __forceinline__ void finish_from_acc(const KParams &p, double *sig_om, double *acc,
+                                                const int *__restrict__ S, int lo, int hi) {
+    for (int i = lo + threadIdx.x; i < hi; i += NT) {
+        const int v = S[i];
+        const double a = __ldcg(&acc[v]);
+        if (ZERO) acc[v] = 0.0;
+        finish_dependency(p, __ldcg(&sig_om[v]), sig_om, v, a);
+    }
+}
+
+template <int NT>
+__device__ __forceinline__ void push_level(const KParams &p, const uint32_t *sw, double *sig_om, double *acc,
+                                           const int *__restrict__ S, int lo, int hi, int hi2, int kpred,
+                                           Counters &c) {
+    // acc is the per-slot omega array, which EP levels of other launches leave dirty
+    for (int i = lo + threadIdx.x; i < hi; i += NT) acc[S[i]] = 0.0;
+    __syncthreads();
+    push_rows<NT, false>(p, sw, sig_om, acc, S, hi, hi2, kpred, 0, NT / 32, c);
+    __syncthreads();
+    finish_from_acc<NT, false>(p, sig_om, acc, S, lo, hi);
+    __syncthreads();
 }
 
 }  // namespace bcdev

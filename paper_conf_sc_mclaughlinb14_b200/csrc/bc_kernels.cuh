@@ -102,6 +102,9 @@ struct KParams {
     int medq;            // fast path: rows in (seq_max_deg, warp_max_deg] are queued and dealt to
                          // warps dynamically after the one-thread rows (graph has such rows)
     int warp_max_deg;    // rows up to this degree: one warp; longer: whole CTA
+    int bpush;           // fast path backward: level L's dependencies are PUSHED from level L+1's
+                         // rows (RED into omega-as-accumulator) when bpush * A_{L+1} < A_L
+                         // (A = arcs of the level's rows); 0 = always pulled (Alg. 3)
     // strategy
     int launch_mode;
     const int *sampled_flag;  // LM_SAMPLED: 1 = EP run
@@ -157,6 +160,8 @@ __device__ __forceinline__ void flush_counters(Counters &c, CtaStats &st) {
     c = Counters{};
 }
 
+constexpr int NLEV_ARCS = 64;  // levels whose arc counts the fast path keeps (deeper: pulled)
+
 template <int NT>
 struct Smem {
     long long idx;
@@ -166,6 +171,7 @@ struct Smem {
     int gw0, gwn;         // row_pass chunk distribution: this CTA's first warp index, warps
                           // sharing the pass (0 / NT/32, except in the group engine's backward)
     int goff;             // group engine: this CTA's offset in the level being compacted
+    unsigned alev[NLEV_ARCS];  // fast path: arcs of the rows of forward level L (L < NLEV_ARCS)
     CtaStats st;
     double red[NT / 32];  // block reduction scratch
     int wtot[NT / 32];    // per-warp totals (frontier compaction)
@@ -988,6 +994,7 @@ bc_kernel(KParams p) {
             ends[1] = 1;
             sm.cnt[0] = sm.cnt[1] = sm.cnt[2] = 0;
         }
+        if (FAST && threadIdx.x < NLEV_ARCS) sm.alev[threadIdx.x] = 0u;
         __syncthreads();
 
         int L = 0, lo = 0, hi = 1;
@@ -1102,16 +1109,23 @@ bc_kernel(KParams p) {
             // the forward's successor bits exist only if forward level Lb ran WE
             uint32_t *const sbl = (sb && (!EPOK || modes[Lb] == MODE_WE)) ? sb : nullptr;
             if constexpr (FAST) {
-                FastLevel f;
-                f.sw = dyn_smem;
-                f.gnb = nullptr;
-                f.sb = nullptr;
-                f.sig = sigma;
-                f.Snext = nullptr;
-                f.cnt = nullptr;
-                f.kmatch = LV::key(Lb + 1);
-                f.knew = 0;
-                fast_pass<NT, false, false>(p, f, S, blo, bhi, Lb, bigq, sm, c, fpass++ & 1);
+                if (p.bpush && Lb + 1 < NLEV_ARCS &&
+                    (unsigned long long)p.bpush * sm.alev[Lb + 1] < (unsigned long long)sm.alev[Lb]) {
+                    // level Lb+1's rows are the cheaper side: push its omega to the predecessors
+                    push_level<NT>(p, dyn_smem, sigma, p.omega + slot * p.stride_n, S, blo, bhi, ends[Lb + 2],
+                                   LV::key(Lb), c);
+                } else {
+                    FastLevel f;
+                    f.sw = dyn_smem;
+                    f.gnb = nullptr;
+                    f.sb = nullptr;
+                    f.sig = sigma;
+                    f.Snext = nullptr;
+                    f.cnt = nullptr;
+                    f.kmatch = LV::key(Lb + 1);
+                    f.knew = 0;
+                    fast_pass<NT, false, false>(p, f, S, blo, bhi, Lb, bigq, sm, c, fpass++ & 1);
+                }
             } else if (!EPOK || bmode == MODE_WE) {
                 backward_we<NT, LV, !EPOK>(p, lv, sigma, S, bigq, sbl, Lb, blo, bhi, sm, c);
             } else {
