@@ -394,7 +394,7 @@ __device__ __forceinline__ void fast_pass(const KParams &p, const FastLevel &f, 
             deg = rows[v + 1] - beg;
         }
         c.scanned += deg;
-        if (FWD && p.bpush && L < NLEV_ARCS) {  // arcs of level L's rows (backward push choice)
+        if (FWD && !G && p.bpush && L < NLEV_ARCS) {  // arcs of level L's rows (backward push choice)
             const unsigned a = __reduce_add_sync(FULL, (unsigned)deg);
             if (lane == 0 && a) atomicAdd(&sm.alev[L], a);
         }
@@ -497,19 +497,15 @@ __device__ __forceinline__ void red_add_f64_if(double *addr, double val, bool c)
 // rows hold most arcs, the level below it few.  The sums are the same up to order (fp64
 // atomics; checked at 1e-9).  S[lo, hi) = level L, S[hi, hi2) = level L+1.  Ends with a
 // barrier.
-// Pushes of the rows S[lo2, hi2) (level L+1) by warps gw0 + wid of gwn; G: global codes.
-template <int NT, bool G>
+// Pushes of the rows S[lo2, hi2) (level L+1) by warps gw0 + wid of gwn; codes in shared memory.
+template <int NT>
 __device__ __forceinline__ void push_rows(const KParams &p, const uint32_t *sw, const double *sig_om, double *acc,
                                           const int *__restrict__ S, int lo2, int hi2, int kpred, int gw0, int gwn,
                                           Counters &c) {
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const int *__restrict__ rows = p.ro;
     const int *__restrict__ cols = p.col;
-    auto code = [&](int u) -> int {
-        if (!G) return code_at(sw, u);
-        const uint32_t wd = __ldca(&sw[(unsigned)u >> 4]);  // codes are final in the backward
-        return (int)(__funnelshift_r(wd, wd, (unsigned)u << 1) & 3u);
-    };
+    auto code = [&](int u) -> int { return code_at(sw, u); };
     for (int base = lo2 + (gw0 + wid) * 32; base < hi2; base += gwn * 32) {
         const int i = base + lane;
         int v = -1, beg = 0, end = 0;
@@ -551,15 +547,13 @@ __device__ __forceinline__ void push_rows(const KParams &p, const uint32_t *sw, 
     }
 }
 
-// Finish of the level-L vertices S[lo, hi) from their pushed sums (acc zeroed after use
-// when ZERO, so the array is clean for the next pushed level).
-template <int NT, bool ZERO>
+// Finish of the level-L vertices S[lo, hi) from their pushed sums.
+template <int NT>
 __device__ __forceinline__ void finish_from_acc(const KParams &p, double *sig_om, double *acc,
                                                 const int *__restrict__ S, int lo, int hi) {
     for (int i = lo + threadIdx.x; i < hi; i += NT) {
         const int v = S[i];
         const double a = __ldcg(&acc[v]);
-        if (ZERO) acc[v] = 0.0;
         finish_dependency(p, __ldcg(&sig_om[v]), sig_om, v, a);
     }
 }
@@ -571,9 +565,9 @@ __device__ __forceinline__ void push_level(const KParams &p, const uint32_t *sw,
     // acc is the per-slot omega array, which EP levels of other launches leave dirty
     for (int i = lo + threadIdx.x; i < hi; i += NT) acc[S[i]] = 0.0;
     __syncthreads();
-    push_rows<NT, false>(p, sw, sig_om, acc, S, hi, hi2, kpred, 0, NT / 32, c);
+    push_rows<NT>(p, sw, sig_om, acc, S, hi, hi2, kpred, 0, NT / 32, c);
     __syncthreads();
-    finish_from_acc<NT, false>(p, sig_om, acc, S, lo, hi);
+    finish_from_acc<NT>(p, sig_om, acc, S, lo, hi);
     __syncthreads();
 }
 

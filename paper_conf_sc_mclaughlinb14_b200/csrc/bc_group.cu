@@ -51,7 +51,6 @@ __device__ __forceinline__ void group_sync(unsigned long long *bar, unsigned lon
 // Levels whose per-CTA share is remembered for the backward (deeper levels -- only on
 // graphs of diameter > RCAP -- are cut in 32-vertex chunks over the whole group).
 constexpr int RCAP = 1024;
-constexpr int GLEV = 24;  // levels whose group-wide arc counts are kept (ctl words 20..31)
 struct Owned {
     const uint32_t *nb;
     int words, r, C, OB, H, items;
@@ -156,7 +155,6 @@ group_kernel(KParams p, GParams gp) {
     unsigned long long *bar = ctl;
     long long *next_idx = reinterpret_cast<long long *>(ctl + 8);
     int *lvl = reinterpret_cast<int *>(ctl + 16);  // level counts, ring of 4
-    unsigned *garcs = reinterpret_cast<unsigned *>(ctl + 20);  // FASTG: arcs of level L's rows, L < GLEV
     GlobalCodes lv;
     lv.w = p.gcodes + (size_t)g * p.stride_codes;
     lv.fb = nullptr;
@@ -215,8 +213,6 @@ group_kernel(KParams p, GParams gp) {
         if (p.perm) s = p.perm[s];
         const long long tsrc = clock64();
         // Alg. 1 by rank 0; every other entry is already unvisited / zero.
-        if (FASTG && tid < NLEV_ARCS) sm.alev[tid] = 0u;
-        if (r == 0 && tid < GLEV) garcs[tid] = 0u;  // every CTA added last source's before its end barrier
         if (r == 0 && tid == 0) {
             lv.set_source(s);
             sigma[s] = 1.0;
@@ -226,7 +222,7 @@ group_kernel(KParams p, GParams gp) {
             lvl[0] = 1;
             lvl[1] = 0;
         }
-        if constexpr (THIN || FASTG) __syncthreads();  // Alg. 1 stores above, read by other lanes below
+        if constexpr (THIN) __syncthreads();  // Alg. 1 stores above, read by other lanes below
         int mylo = 0, mycnt = r == 0 ? 1 : 0;  // this CTA's vertices of level L: S[mylo, +mycnt)
         if (tid == 0) s_reg[0] = make_int2(mylo, mycnt);
         int prevlo = 0, prevcnt = 0;
@@ -248,7 +244,6 @@ group_kernel(KParams p, GParams gp) {
                     fast_pass<NT, true, true>(p, mk(nbw_next, GlobalCodes::key(L - 1), GlobalCodes::key(L + 1)), S,
                                               mylo, mylo + mycnt, L, bigq, sm, c, fpass++ & 1);
                     c.arcs_reached += c.scanned - before;
-                    if (p.bpush && tid == 0 && L < GLEV && L < NLEV_ARCS && sm.alev[L]) atomicAdd(&garcs[L], sm.alev[L]);
                 }
             }
             // (b) level L+1 is complete once every CTA got here
@@ -309,23 +304,7 @@ group_kernel(KParams p, GParams gp) {
         // ownership, same locality); levels >= RCAP in 32-vertex chunks over the group.
         for (int Lb = maxdepth - 1; Lb >= 1; --Lb) {
             const long long t0 = clock64();
-            bool pushed = false;
-            if constexpr (FASTG) {
-                if (p.bpush && Lb + 1 < GLEV && Lb + 1 < RCAP &&
-                    (unsigned long long)p.bpush * __ldcg(&garcs[Lb + 1]) < (unsigned long long)__ldcg(&garcs[Lb])) {
-                    // level Lb+1's rows are the cheaper side: its owners push omega to the
-                    // predecessors, then each CTA finishes its own level-Lb vertices
-                    const int2 r1 = s_reg[Lb + 1];
-                    push_rows<NT, true>(p, lv.w, sigma, p.omega + (size_t)g * p.stride_n, S, r1.x, r1.x + r1.y,
-                                        GlobalCodes::key(Lb), 0, NW, c);
-                    group_sync(bar, target, C, &sm.st.gwait);
-                    const int2 rg = s_reg[Lb];
-                    finish_from_acc<NT, true>(p, sigma, p.omega + (size_t)g * p.stride_n, S, rg.x, rg.x + rg.y);
-                    pushed = true;
-                }
-            }
-            if (pushed) {
-            } else if (Lb < RCAP) {
+            if (Lb < RCAP) {
                 const int2 rg = s_reg[Lb];
                 if constexpr (THIN) {
                     thin_pass<NT, false>(p, tl_(nullptr, GlobalCodes::key(Lb + 1), 0), S, rg.x, rg.x + rg.y, Lb, bigq,
