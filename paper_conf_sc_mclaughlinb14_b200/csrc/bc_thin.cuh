@@ -1,16 +1,19 @@
-// bc_thin.cuh -- thin-row level passes of the group engine: the same
+// bc_thin.cuh -- thin-row level passes of the group engine (DESIGN.md §5c'): the same
 // forward (Alg. 2 l.3-8 as a pull) and backward (Alg. 3 l.5-9 with the omega
-// trick; Eq. 3) as forward_we / backward_we, for graphs whose rows are
-// short and even (no hubs: c5ws, the Watts-Strogatz small world, degree ~10).
+// trick; Eq. 3) as forward_we / backward_we, for large graphs whose rows
+// are short and even (no hubs: c5ws, the Watts-Strogatz small world, degree ~10).
 //
-// One row per VIRTUAL warp of VW lanes (Hong et al.'s virtual warps) instead of one row per
-// thread: lane t of a row's VW lanes takes arcs t, t + VW, ... with U arcs in flight per
-// iteration (U independent col -> code -> sigma chains per lane), so a warp keeps 32 U arcs
-// in flight with every lane busy, where a thread-per-row quad loop leaves lanes idle at row
-// ends (ncu r02: SIMT efficiency 0.67, 3 warp instructions per scanned arc).  The per-row
-// sum is reduced over the VW lanes (a different order of additions than the CSR order:
-// sigma sums of integers below 2^53 are exact in any order, omega sums are checked at 1e-9).
-// Rows longer than THIN_MAX are queued and expanded by a whole warp each afterwards.
+// Each row is taken by VW lanes (default 1: one row per lane); every lane runs U independent
+// col -> code -> sigma chains per iteration (arcs t, t + VW, ..., t + (U-1) VW of its slice),
+// the iteration count is warp-uniform, and the S entries / row bounds of the lane's next
+// chunk are loaded while the current chunk is expanded.  Against the generic row_pass
+// (aligned quads, 3-4 sequential probe -> gather rounds per row, SIMT efficiency 0.67,
+// spills at the 64-register cap) this measured 1503 -> 1416 ms per 2,048 c5ws sources on
+// B200; virtual warps of 2/4/8 lanes per row (Hong et al.) keep fewer rows in flight and
+// were slower (profiles/r02/ab/thin_rows.txt).  With VW > 1 the per-row sum is reduced over
+// the VW lanes (a different order of additions: sigma sums of integers below 2^53 are exact
+// in any order, omega sums are checked at 1e-9).  Rows longer than THIN_MAX are queued and
+// expanded by a whole warp each afterwards.
 //
 // Level codes are the group engine's global 2-bit codes (GlobalCodes: 0 unvisited,
 // 1 + L mod 3), read through L1 (invalidated at every group barrier).  Discoveries are
@@ -53,9 +56,9 @@ __device__ __forceinline__ int gcode(const uint32_t *codes, int u) {
     return (int)(__funnelshift_r(wd, wd, (unsigned)u << 1) & 3u);
 }
 
-// Forward arcs a0 + j*S + t (j < U) of a row ending at e, for lanes t of a group of S lanes
-// sharing the row (S = VW, or 32 for a wide row).  Accumulates the pull sum into acc and
-// returns the successor slices (bit j*S' .. of the group's ballots) through succ[j].
+// Forward arcs a0 + j * stride (j < U; a0 already includes the lane's offset in its row) of a
+// row ending at e (stride = VW, or 32 for a wide row).  Adds the pull sum to acc, counts the
+// DAG (predecessor) arcs, and returns the warp ballot of successor arcs of slot j in succm[j].
 template <int U>
 __device__ __forceinline__ void thin_fwd_step(const ThinLevel &t, int a0, int e, int stride, double &acc,
                                               unsigned &dag, unsigned (&succm)[U]) {
