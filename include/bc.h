@@ -96,7 +96,9 @@ typedef struct bc_options {
     int32_t backward_we;     /* 1: backward always WE (Alg. 3); 0 (default): backward level L
                                 uses the mode forward level L used (R8)              */
     /* Implementation knobs (do not change results beyond fp64 rounding order): */
-    int32_t block_threads;   /* threads per CTA: 0 = auto, 128, 256, 512 or 1024                */
+    int32_t block_threads;   /* threads per CTA: 0 = auto (128 below 2^17 vertices, else 512;
+                                1024 for degree-relabelled graphs with codes in shared memory),
+                                128, 256, 512 or 1024                                          */
     int32_t seq_max_deg;     /* rows up to this degree are summed by one thread in CSR order;
                                 longer rows cooperatively.  0 = auto (128)                     */
     int32_t level_store;     /* 0 = auto, 1 = exact int32 d in HBM, 2 = 2-bit codes in shared
@@ -104,8 +106,9 @@ typedef struct bc_options {
                                 3 = 2-bit codes in HBM/L2 (undirected graphs)                  */
     int32_t warp_max_deg;    /* rows up to this degree are expanded by one warp, longer rows
                                 by the whole CTA.  0 = auto (8192)                             */
-    int32_t l2_persist;      /* 0 = auto (on), -1 = off: persisting-L2 access-policy window
-                                over the CSR arrays during traversal launches                  */
+    int32_t l2_persist;      /* 0 = auto, 1 = on, -1 = off: persisting-L2 access-policy window
+                                over the CSR arrays during traversal launches (auto: on, except
+                                for degree-relabelled graphs with level codes in shared memory) */
     int32_t sort_frontier;   /* 0 = auto, 1 = on, -1 = off: rebuild large BFS levels in vertex
                                 order from a per-level bitmap (locality of rows, codes, sigma)  */
     /* Output post-processing (default 0 = exact BC as defined above): */

@@ -270,6 +270,9 @@ static int configure(bc_graph *g) {
         // 10^3..10^5 vertices, hub rows) want wide CTAs; small graphs want many
         // narrow ones (frontiers of a few hundred vertices, more roots in flight).
         nt = g->n >= (1 << 17) ? 512 : 128;
+        // degree-relabelled (skewed) graphs since the backward push: 1,024 threads, one
+        // source per SM (c4: 487 -> 466 ms per 16,384 sources; c3, unskewed, 227 -> 286 ms)
+        if (g->perm && g->n >= (1 << 17) && g->lstore == 2) nt = 1024;
     }
     if (nt != 128 && nt != 256 && nt != 512 && nt != 1024)
         return fail(BC_EINVAL, "block_threads must be 0, 128, 256, 512 or 1024");
@@ -299,11 +302,15 @@ static int configure(bc_graph *g) {
     // Persisting-L2 window over the CSR (plus src[] when EP levels can run): every
     // in-flight source re-reads the same rows, while sigma/omega gathers stream.
     g->l2win = cudaAccessPolicyWindow{};
-    if (o.l2_persist < 0 && g->l2_held) {  // window switched off: stop holding the carve-out
+    // auto: on, except for skewed graphs on the shared-memory-codes engine, whose CSR reads
+    // hit L2 anyway once fewer sources are in flight (c4 at 1,024 threads: 466 -> 460 ms
+    // without the window; c3 / c2d neutral)
+    const bool l2_on = o.l2_persist > 0 || (o.l2_persist == 0 && !(g->perm && g->lstore == 2));
+    if (!l2_on && g->l2_held) {  // window switched off: stop holding the carve-out
         l2_release(g->device);
         g->l2_held = false;
     }
-    if (o.l2_persist >= 0 && g->graph_buf) {
+    if (l2_on && g->graph_buf) {
         int max_persist = 0, max_win = 0;
         CK(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, g->device));
         CK(cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, g->device));

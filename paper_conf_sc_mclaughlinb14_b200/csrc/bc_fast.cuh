@@ -141,6 +141,53 @@ __device__ __forceinline__ uint64_t sb_window(const uint32_t *sb, int w0, int en
     return win;
 }
 
+// Backward sum of one row [beg, end) over its successor arcs only, taken from the
+// successor bitmap four at a time (find-first-set on a 64-arc window): the columns and
+// omega gathers of up to four successors are issued together, so a row costs one window
+// load + one column round trip + one gather round trip per four successors, whatever its
+// length (the quad walk paid a loop trip per four arcs).  Sums in CSR order.
+#ifndef BC_SUCC_EXTRACT
+#define BC_SUCC_EXTRACT 1
+#endif
+__device__ __forceinline__ double succ_sum(const uint32_t *sb, const int *__restrict__ cols, const double *sig,
+                                           int beg, int end) {
+    double acc = 0.0;
+    if (end <= beg) return acc;
+    int base = (beg >> 5) << 5;  // window [base, base + 64)
+    auto window = [&](int b) -> uint64_t {
+        uint64_t w = __ldcg(&sb[b >> 5]);
+        if (end > b + 32) w |= (uint64_t)__ldcg(&sb[(b >> 5) + 1]) << 32;
+        if (end - b < 64) w &= (1ull << (end - b)) - 1ull;
+        return w;
+    };
+    uint64_t win = window(base) & (~0ull << (beg - base));
+    for (;;) {
+        int a[4];
+        bool ok[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            while (win == 0ull && base + 64 < end) {  // rows longer than the window
+                base += 64;
+                win = window(base);
+            }
+            ok[j] = win != 0ull;
+            a[j] = base + (ok[j] ? __ffsll((long long)win) - 1 : 0);
+            win &= win - 1ull;
+        }
+        if (!ok[0]) break;
+        int u[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) u[j] = ok[j] ? ld_col(cols + a[j]) : 0;
+        double g[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) g[j] = ldca_if(sig + u[j], ok[j]);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc += g[j];
+        if (!ok[3]) break;
+    }
+    return acc;
+}
+
 // Quads of the one-thread rows of a 32-vertex chunk; lane = row [beg, end) (deg <= seq_max,
 // deg = 0 for lanes without a row).  Warp-uniform trip count.  Returns the lane's sum of
 // gathers in CSR order.
@@ -156,6 +203,7 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
         // backward: only the successor arcs the forward marked; no probe
         // (per-lane trip count: no warp collective in here, and a lane whose quads hold no
         // successor skips them)
+        if (BC_SUCC_EXTRACT) return succ_sum(f.sb, cols, f.sig, beg, end);
         int w0 = beg >> 5;
         uint64_t win = sb_window(f.sb, w0, end, nq > 0);
         for (int q = 0; q < nq; ++q) {

@@ -200,10 +200,14 @@ __device__ BC_THIN_INL void thin_pass(const KParams &p, const ThinLevel &t, cons
                 red_or_global_if(&t.sb[(wbase >> 5) + 1], (uint32_t)(win >> 32), (win >> 32) != 0ull);
             }
         } else {
-            const uint64_t win = end > beg ? sb_pair(t.sbr, wbase >> 5, end > wbase + 32) : 0ull;
-            for (int it = 0; it < maxit; ++it) {
-                const int a0 = beg + it * VW * U;
-                acc += thin_bwd_step<U>(t, a0 + sub, end, VW, win, wbase);
+            if (VW == 1 && BC_SUCC_EXTRACT) {  // the row's successors, four at a time
+                acc = succ_sum(t.sbr, t.col, t.sig, beg, end);
+            } else {
+                const uint64_t win = end > beg ? sb_pair(t.sbr, wbase >> 5, end > wbase + 32) : 0ull;
+                for (int it = 0; it < maxit; ++it) {
+                    const int a0 = beg + it * VW * U;
+                    acc += thin_bwd_step<U>(t, a0 + sub, end, VW, win, wbase);
+                }
             }
         }
 #pragma unroll
