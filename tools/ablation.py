@@ -76,7 +76,7 @@ def main():
     import paper_conf_sc_mclaughlinb14_b200 as bcm
     from paper_conf_sc_mclaughlinb14_b200 import graphgen as gg
     rows = []
-    head = os.popen("git rev-parse --short HEAD 2>/dev/null").read().strip() or None
+    head = os.environ.get("BC_HEAD") or os.popen("git rev-parse --short HEAD 2>/dev/null").read().strip() or None
 
     def run(g, key, src, d_src, out, strategy, sweep, label, value, opts):
         bg = bcm.BCGraph.from_graph(g, strategy=strategy, **opts)
