@@ -515,7 +515,8 @@ static int group_mode(const bc_graph *g) {
 
 static int alloc_group(bc_graph *g) {
     bc_graph::Group &q = g->gr;
-    const int nt = g->n >= (1 << 17) ? 512 : 256;
+    int nt = g->n >= (1 << 17) ? 512 : 256;
+    if (const char *e = getenv("BC_GROUP_NT")) nt = atoi(e);  // tuning override (1024: tuning build)
     int per_sm = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bcgroup::group_kernel_fn(nt, group_mode(g)), nt, 0));
     if (per_sm < 1) return fail(BC_EINTERNAL, "group kernel cannot be resident");

@@ -138,7 +138,7 @@ __device__ __forceinline__ int group_compact(uint32_t *nb, int words, int r, int
 #define BC_THIN_MINB 2
 #endif
 template <int NT, int MODE>
-__global__ void __launch_bounds__(NT, NT >= 512 ? (MODE == GM_THIN ? BC_THIN_MINB : 2) : 4)
+__global__ void __launch_bounds__(NT, NT >= 1024 ? 1 : NT >= 512 ? (MODE == GM_THIN ? BC_THIN_MINB : 2) : 4)
 group_kernel(KParams p, GParams gp) {
     constexpr bool FASTG = MODE == GM_FAST;
     constexpr bool THIN = MODE == GM_THIN;
@@ -389,6 +389,13 @@ group_kernel(KParams p, GParams gp) {
 }
 
 const void *group_kernel_fn(int nt, int mode) {
+#if defined(BC_GROUP_1024) && BC_GROUP_1024
+    if (nt == 1024) {  // tuning build only (BC_GROUP_NT=1024)
+        if (mode == GM_FAST) return (const void *)group_kernel<1024, GM_FAST>;
+        if (mode == GM_THIN) return (const void *)group_kernel<1024, GM_THIN>;
+        return (const void *)group_kernel<1024, GM_GENERIC>;
+    }
+#endif
     if (mode == GM_FAST) return nt == 256 ? (const void *)group_kernel<256, GM_FAST> : (const void *)group_kernel<512, GM_FAST>;
     if (mode == GM_THIN) return nt == 256 ? (const void *)group_kernel<256, GM_THIN> : (const void *)group_kernel<512, GM_THIN>;
     return nt == 256 ? (const void *)group_kernel<256, GM_GENERIC> : (const void *)group_kernel<512, GM_GENERIC>;
