@@ -141,6 +141,23 @@ __device__ __forceinline__ uint64_t sb_window(const uint32_t *sb, int w0, int en
     return win;
 }
 
+// acc + g[0] + g[1] + g[2] + g[3] in CSR order.  (BC_TREE_ADD=1, a tuning build: as
+// acc + ((g0 + g1) + (g2 + g3)), one dependent DADD per quad on the accumulator instead of
+// four -- measured neutral on B200: c4 460.0 -> 460.5 ms, c2d 251.2 -> 254.1, c5k 1921 ->
+// 1908; not kept, the CSR order stays.)
+#ifndef BC_TREE_ADD
+#define BC_TREE_ADD 0
+#endif
+__device__ __forceinline__ double add4(double acc, const double (&g)[4]) {
+#if BC_TREE_ADD
+    return acc + ((g[0] + g[1]) + (g[2] + g[3]));
+#else
+#pragma unroll
+    for (int j = 0; j < 4; ++j) acc += g[j];
+    return acc;
+#endif
+}
+
 // Backward sum of one row [beg, end) over its successor arcs only, taken from the
 // successor bitmap four at a time (find-first-set on a 64-arc window): the columns and
 // omega gathers of up to four successors are issued together, so a row costs one window
@@ -181,8 +198,7 @@ __device__ __forceinline__ double succ_sum(const uint32_t *sb, const int *__rest
         double g[4];
 #pragma unroll
         for (int j = 0; j < 4; ++j) g[j] = ldca_if(sig + u[j], ok[j]);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc += g[j];
+        acc = add4(acc, g);
         if (!ok[3]) break;
     }
     return acc;
@@ -224,8 +240,7 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
             double g[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) g[j] = ldca_if(f.sig + u[j], (sbits >> j) & 1u);
-#pragma unroll
-            for (int j = 0; j < 4; ++j) acc += g[j];
+            acc = add4(acc, g);
         }
         return acc;
     }
@@ -278,8 +293,7 @@ __device__ __forceinline__ double fast_seq_rows(const FastLevel &f, const int *_
                 win |= (uint64_t)sm4 << off;
             }
         }
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc += g[j];
+        acc = add4(acc, g);
     }
     if (FWD && bits) sb_flush(f.sb, w0, win);
     if (FWD) c.dag += dag;
@@ -328,8 +342,7 @@ __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *_
             double g[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) g[j] = ldca_if(f.sig + u[j], s[j]);
-#pragma unroll
-            for (int j = 0; j < 4; ++j) acc += g[j];
+            acc = add4(acc, g);
         }
         return acc;
     }
@@ -387,14 +400,11 @@ __device__ __forceinline__ double fast_coop_row(const FastLevel &f, const int *_
                 }
             }
         }
+        acc = add4(acc, gp);
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            acc += gp[j];
-            gp[j] = g[j];
-        }
+        for (int j = 0; j < 4; ++j) gp[j] = g[j];
     }
-#pragma unroll
-    for (int j = 0; j < 4; ++j) acc += gp[j];
+    acc = add4(acc, gp);
     if (FWD) c.dag += dag;
     return acc;
 }
