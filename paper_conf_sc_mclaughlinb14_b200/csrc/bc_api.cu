@@ -1112,7 +1112,40 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
     const int mode_main = strat == BC_STRATEGY_WE ? LM_WE : strat == BC_STRATEGY_EP ? LM_EP
                         : strat == BC_STRATEGY_HYBRID ? LM_HYBRID : LM_SAMPLED;
     long long ks = 0;
-    if (strat == BC_STRATEGY_SAMPLING) {
+    // Alg. 5 with a guard no frontier can reach (ep_min_frontier > n, the bench's B200
+    // guard): the decision cannot change how any source runs (every level is WE either
+    // way), so the sampling sources and the rest go in ONE launch -- the first n_samps still
+    // record their max depth and the decision is still taken and reported afterwards --
+    // instead of two launches with a tail each (c1: two waves of 512 sources -> one).
+    const bool merged = strat == BC_STRATEGY_SAMPLING && (long long)g->opt.ep_min_frontier > (long long)g->n &&
+                        !batch_wanted(g) && !getenv("BC_NO_MERGE");
+    if (merged) {
+        ks = std::min<long long>(k, g->opt.n_samps);
+        KParams pm = p;
+        pm.launch_mode = LM_WE;
+        pm.src_base = 0;
+        pm.k = k;
+        pm.keys = g->keys;
+        pm.nkeys = ks;
+        pm.work_counter = g->counters + 1;
+        if (k > 0) {
+            CK(cudaEventRecord(g->tev[2], st));
+            if ((rc = launch(g, pm, st))) return rc;
+            CK(cudaEventRecord(g->tev[3], st));
+            g->tev_used[1] = 1;
+        }
+        if (ks > 0) {
+            int P = 1;
+            while (P < ks) P <<= 1;
+            const double thresh = g->opt.gamma * std::log2((double)std::max(g->n, 1));
+            sampling_decide_kernel<<<1, 1024, sizeof(int) * (size_t)P, st>>>(g->keys, (int)ks, thresh,
+                                                                           g->flag, g->stats);
+            CK(cudaGetLastError());
+            g->launches++;
+            g->sampling_ran = 1;
+        }
+        ks = k;  // nothing left for the main phase below
+    } else if (strat == BC_STRATEGY_SAMPLING) {
         // Alg. 5: first n_samps sources WE, record max depth, decide, then the rest.
         ks = std::min<long long>(k, g->opt.n_samps);
         KParams ps = p;
@@ -1120,6 +1153,7 @@ static int enqueue_compute(bc_graph *g, const int *d_sources, long long k, doubl
         ps.src_base = 0;
         ps.k = ks;
         ps.keys = g->keys;
+        ps.nkeys = ks;
         ps.work_counter = g->counters;
         if (ks > 0) {
             CK(cudaEventRecord(g->tev[0], st));

@@ -280,7 +280,7 @@ group_kernel(KParams p, GParams gp) {
         const int maxdepth = L - 1;
         const int S_len = startL;
         const long long tfwd = clock64();
-        if (p.keys && r == 0 && tid == 0) p.keys[idx] = maxdepth;
+        if (p.keys && idx < p.nkeys && r == 0 && tid == 0) p.keys[idx] = maxdepth;
         if (p.dbg_d) {  // debug export of d and sigma before omega overwrites sigma
             for (int l = 0; l <= maxdepth; ++l) {
                 const int lo = ends[l], hi = ends[l + 1];

@@ -110,7 +110,8 @@ struct KParams {
     const int *sampled_flag;  // LM_SAMPLED: 1 = EP run
     int alpha, beta, ep_min_frontier;
     int backward_we;
-    int *keys;                // sampling phase: keys[idx] = max depth
+    int *keys;                // sampling phase: keys[idx] = max depth, for idx < nkeys
+    long long nkeys;
     DevStats *stats;
     // debug export (single source), may be NULL
     int *dbg_d;
@@ -1085,7 +1086,7 @@ bc_kernel(KParams p) {
         }
         const int maxdepth = L;
         const int S_len = hi;
-        if (p.keys && threadIdx.x == 0) p.keys[idx] = maxdepth;
+        if (p.keys && idx < p.nkeys && threadIdx.x == 0) p.keys[idx] = maxdepth;
 
         if (p.dbg_d) {  // debug export of d and sigma before omega overwrites sigma
             for (int l = 0; l <= maxdepth; ++l)
